@@ -1,0 +1,313 @@
+#!/usr/bin/env python
+"""Benchmark: verified GB/s (both arrays read) of the kernel-verification comparison.
+
+Workload (BASELINE.json configs[3], the config the metric's "1/2/4/8 B200" is
+quoted on): C4 -- fp64, 2^29 elements per array (4 GiB each, 8 GiB read per
+step), 512 injected mismatches + 4 NaN/number pairs, abs_tol 1e-6, rel_tol
+1e-5, max_report 2^20.  At N GPUs the array is split into N contiguous shards
+(one per rank, generated on that rank) and every step is one collective
+arc_verify_compare (local kernel + NCCL merge): strong scaling, fixed total.
+
+One step = one arc_verify_compare call on HBM-resident arrays (the whole hot
+path: stream + predicate + reductions + ordered compaction + summary/report to
+the host).  value = global bytes (2 * n * 8) * K / max-over-ranks device time.
+e2e = the same metric through the same C-ABI call with the arrays in pinned
+HOST memory: the library streams them to the GPU in chunks overlapped with the
+comparison, so H2D copies are inside the timed region.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+N_C4 = 1 << 29
+ES = 8
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--n", type=int, default=N_C4, help="elements per array (default: C4's 2^29)")
+    ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--profile", action="store_true", help="short run for ncu (no clocks/e2e/cpu)")
+    return ap.parse_args()
+
+
+def measured_peak():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(path) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy r+w)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+def ncu_traffic():
+    """dram bytes (read+write) per launch of the compare kernel from the committed ncu capture."""
+    path = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        with open(path) as f:
+            d = json.load(f)
+        return d.get("c4_dram_bytes_per_launch")
+    except Exception:
+        return None
+
+
+class ClockSampler:
+    """Samples SM clock and throttle reasons via NVML while the timed region runs."""
+
+    REASONS = {
+        0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+        0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+        0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting",
+    }
+
+    def __init__(self, device: int):
+        self.samples, self.reasons, self.ok = [], set(), False
+        self.max_mhz = None
+        try:
+            import pynvml
+
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(device)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # pragma: no cover
+            self.err = str(e)
+        self._stop = threading.Event()
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                fn = getattr(self.nv, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
+                    self.nv.nvmlDeviceGetCurrentClocksThrottleReasons
+                mask = fn(self.h)
+                for bit, name in self.REASONS.items():
+                    if mask & bit and bit != 0x1:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.005)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self.ok:
+            self._stop.set()
+            self.t.join()
+
+    def summary(self):
+        if not self.ok or not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": ["unavailable"], "samples": 0}
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+# ---------------------------------------------------------------- reference
+def run_reference(args, rank):
+    """The oracle, as it stands, on the host cores: each step a bounded sample of C4."""
+    if rank != 0:
+        return
+    import oracle
+    import synth
+
+    oracle.build()
+    sample = 1 << 22
+    c4 = synth.C4(args.n)
+    out, ref = c4.slice(0, min(sample, args.n))
+    o, r = out.numpy(), ref.numpy()
+    for _ in range(args.warmup):
+        oracle.compare(o, r, "f64", c4.abs_tol, c4.rel_tol, c4.max_report)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle.compare(o, r, "f64", c4.abs_tol, c4.rel_tol, c4.max_report)
+    dt = time.perf_counter() - t0
+    gbs = 2 * o.size * ES * args.steps / dt / 1e9
+    line = {
+        "impl": "reference", "metric": "verified GB/s (both arrays read)", "value": round(gbs, 3),
+        "unit": "GB/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(dt / args.steps * 1e3, 3), "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"C4 sample: first {o.size} elements (fp64) of the C4 arrays per step",
+                   "parallelism": "1 host core"},
+        "cpu_baseline": {"value": round(gbs, 3), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                         "sample": f"first 2^22 of 2^29 C4 elements, {args.steps} steps"},
+        "e2e": {"value": round(gbs, 3), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def cpu_baseline(c4, n):
+    """Oracle on the host (1 core) over a bounded C4 sample, ~5 s of CPU work."""
+    import oracle
+
+    oracle.build()
+    sample = min(1 << 24, n)
+    out, ref = c4.slice(0, sample)
+    o, r = out.numpy(), ref.numpy()
+    reps, t_total = 0, 0.0
+    while t_total < 5.0 and reps < 20:
+        t0 = time.perf_counter()
+        oracle.compare(o, r, "f64", c4.abs_tol, c4.rel_tol, c4.max_report)
+        t_total += time.perf_counter() - t0
+        reps += 1
+    gbs = 2 * sample * ES * reps / t_total / 1e9
+    return {"value": round(gbs, 3), "unit": "GB/s", "cores": 1, "kind": "oracle",
+            "sample": f"first 2^24 of the 2^29 C4 elements (fp64), {reps} repetition(s), {t_total:.1f} s"}
+
+
+# --------------------------------------------------------------------- ours
+def main():
+    args = parse()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        return run_reference(args, rank)
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_leelv14_b200 as av
+    import synth
+
+    assert world == args.gpus, f"--gpus {args.gpus} but WORLD_SIZE {world}"
+    torch.cuda.set_device(local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        av.init_distributed()
+    else:
+        av.init(local_rank)
+
+    n = args.n
+    lo, hi = rank * n // world, (rank + 1) * n // world
+    c4 = synth.C4(n)
+    out, ref = c4.slice(lo, hi - lo, device="cuda")
+    torch.cuda.synchronize()
+    mr = c4.max_report
+
+    def step():
+        return av.compare(out, ref, c4.abs_tol, c4.rel_tol, mr)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    for _ in range(args.warmup):
+        res = step()
+    barrier()
+    av.arc_verify_set_timing(True)
+    av.arc_verify_kernel_stats(reset=True)
+    stream = torch.cuda.current_stream()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    sampler = ClockSampler(local_rank) if not args.profile else None
+    barrier()
+    if sampler:
+        sampler.__enter__()
+    ev0.record(stream)
+    for _ in range(args.steps):
+        res = step()
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    if sampler:
+        sampler.__exit__()
+    ms = ev0.elapsed_time(ev1)
+    launches, kern_ms = av.arc_verify_kernel_stats(reset=True)
+    av.arc_verify_set_timing(False)
+    t = torch.tensor([ms, kern_ms / max(launches, 1)], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_max, kern_avg_ms = float(t[0]), float(t[1])
+
+    # parity of the timed result against the generator's closed form
+    planted = c4.planted()
+    parity = (res.n_mismatch == len(planted) and list(res.report["index"]) == planted)
+
+    total_bytes = 2 * n * ES
+    value = total_bytes * args.steps / (ms_max / 1e3) / 1e9
+    local_bytes = 2 * (hi - lo) * ES
+    achieved = local_bytes / (kern_avg_ms / 1e3) / 1e9
+    peak, peak_src = measured_peak()
+
+    # ------------------------------------------------------------------ e2e
+    e2e = None
+    if not args.no_e2e and not args.profile:
+        ho = out.cpu().pin_memory()
+        hr = ref.cpu().pin_memory()
+        del_out = None
+        step_h = lambda: av.compare(ho, hr, c4.abs_tol, c4.rel_tol, mr)  # noqa: E731
+        step_h()
+        barrier()
+        t0 = torch.cuda.Event(enable_timing=True)
+        t1 = torch.cuda.Event(enable_timing=True)
+        t0.record(stream)
+        for _ in range(args.e2e_steps):
+            rh = step_h()
+        t1.record(stream)
+        torch.cuda.synchronize()
+        te = torch.tensor([t0.elapsed_time(t1)], dtype=torch.float64, device="cuda")
+        if world > 1:
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        e2e_ms = float(te[0])
+        parity = parity and rh.n_mismatch == res.n_mismatch
+        e2e = {"value": round(total_bytes * args.e2e_steps / (e2e_ms / 1e3) / 1e9, 3), "unit": "GB/s",
+               "h2d_bytes_per_step": 2 * (hi - lo) * ES * world,
+               "d2h_bytes_per_step": (32 + 24 * rh.n_reported) * world,
+               "steps": args.e2e_steps, "ms_per_step": round(e2e_ms / args.e2e_steps, 3),
+               "path": "arc_verify_compare with pinned host out/ref (chunked H2D overlapped with compare)"}
+        del ho, hr, del_out
+
+    if rank == 0:
+        line = {
+            "metric": "verified GB/s (both arrays read)",
+            "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(ms_max / args.steps, 4), "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": "C4: fp64 2^29 elements per array (4 GiB each), 512 injected + 4 NaN "
+                                   "pairs, abs_tol 1e-6, rel_tol 1e-5, max_report 2^20",
+                       "n": n, "parallelism": f"shard{world}" if world > 1 else "single",
+                       "l2": "inputs (8 GiB) larger than L2 (126 MB); no flush",
+                       "report": "host (numpy) buffer"},
+            "parity": "ok" if parity else "FAIL",
+            "gpu_launches": int(launches) + (args.steps if world > 1 else 0),
+            "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                         "frac": round(achieved / peak, 4), "traffic": ncu_traffic(),
+                         "kernel": "arcv_compare_kernel", "kernel_ms_avg": round(kern_avg_ms, 4),
+                         "algorithmic_bytes_per_launch": local_bytes, "peak_source": peak_src},
+            "e2e": e2e,
+        }
+        if sampler:
+            line["clocks"] = sampler.summary()
+        if world == 1 and not args.no_cpu_baseline and not args.profile:
+            line["cpu_baseline"] = cpu_baseline(c4, n)
+        print(json.dumps(line), flush=True)
+    av.finalize()
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,252 @@
+/*
+ * arc_verify.h -- C ABI of the B200-native kernel-verification result comparison.
+ *
+ * The operation (PAPER.md = /root/reference/PAPER.md, cited as P:<line>):
+ *   sec. III-A, P:159  "we propose to compare these results at the granularity of
+ *                       a GPU kernel": the outputs of a translated GPU region are
+ *                       compared with the outputs of the sequential CPU region.
+ *   sec. III-A, P:171  "all data modified by the kernel are copied back to a
+ *                       temporary space on the CPU after the kernel finished";
+ *                       Listing 2 line 11: "Result comparison codes
+ *                       will be added" after "#pragma acc wait(1)".
+ *   sec. III-A, P:199  "If the output difference is bigger than the allowed error
+ *                       margin, then an error will be reported to the user ...
+ *                       the transformation allows users to configure the error
+ *                       margin".
+ *   sec. III-A, P:161  the margin exists because "CPU and GPU may use different
+ *                       numbers of bits to store floating-point numbers, and
+ *                       non-deterministic computation order".
+ * This library runs the comparison itself on the GPU (the paper ran it on the
+ * host CPU over data copied back over PCIe), so only the
+ * summary and the report cross to the host.
+ *
+ * Per element i, for float dtypes (x = (double)out[i], y = (double)ref[i],
+ * exact widening; arithmetic in IEEE fp64, round-to-nearest, no FMA contraction,
+ * no flush-to-zero):
+ *   rule 1  x == y                -> match, d = 0, r = 0        (covers +-0, equal Inf)
+ *   rule 2  isnan(x) && isnan(y)  -> match, d and r excluded from the maxima
+ *   rule 3  isnan(x) || isnan(y)  -> mismatch, d and r excluded
+ *   rule 4  isinf(y)              -> mismatch, d = r = +Inf
+ *   rule 5  d = |x - y|, t = abs_tol + (rel_tol * |y|) as two rounded operations;
+ *           match iff d <= t; r = d / |y| (+Inf if d = +Inf or y = 0)
+ * For integer dtypes: match iff out[i] == ref[i] (tolerances ignored);
+ * d = |out[i] - ref[i]| computed exactly and converted to double (RN); no r.
+ * The readings behind rules 1-5 (the paper gives no formula) are DESIGN.md
+ * sec. 3, R1-R12.
+ *
+ * Result: n_mismatch = exact count; max_abs_err / max_rel_err = max of the
+ * defined d / r (0 if none; max_rel_err = 0 for integers); report = the first
+ * max_report mismatches in ascending index order, each (index, raw bits of
+ * out[i], raw bits of ref[i]) zero-extended to 64 bits.  The GPU result is
+ * bit-identical to the CPU oracle (oracle/arc_oracle.c) for any launch geometry,
+ * batching or sharding.
+ *
+ * Conventions
+ *  - Every call returns an arc_status_t.  A mismatch is data, not an error
+ *    (ARC_OK with n_mismatch > 0).
+ *  - One context per process; calls are not thread-safe (the caller serialises).
+ *  - Work is enqueued on the stream given at init (or arc_verify_set_stream) and
+ *    every call returns after its result is on the host (the paper's
+ *    "acc wait" before comparison, Listing 2 line 10).
+ *  - Ownership: the library never owns or frees caller arrays or report
+ *    buffers; it owns its workspace (look-back status words, accumulators,
+ *    staging), allocated lazily, grown on demand, freed by arc_verify_finalize.
+ */
+#ifndef ARC_VERIFY_H
+#define ARC_VERIFY_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    ARC_OK = 0,
+    ARC_E_INVAL = -1,       /* bad argument (see each call)                        */
+    ARC_E_NOINIT = -2,      /* called before arc_verify_init                       */
+    ARC_E_CUDA = -3,        /* a CUDA runtime call failed (text: arc_verify_last_error) */
+    ARC_E_NCCL = -4,        /* an NCCL call failed, or NCCL could not be loaded    */
+    ARC_E_NOMEM = -5,       /* workspace allocation failed                         */
+    ARC_E_UNSUPPORTED = -6  /* valid request this build does not support           */
+} arc_status_t;
+
+typedef enum { ARC_F32 = 0, ARC_F64 = 1, ARC_I32 = 2, ARC_I64 = 3, ARC_U8 = 4 } arc_dtype_t;
+
+/* One reported mismatch: 24 bytes, raw bit patterns zero-extended. */
+typedef struct {
+    uint64_t index;    /* element index (global index when sharded)  */
+    uint64_t out_bits; /* raw bits of out[index]                     */
+    uint64_t ref_bits; /* raw bits of ref[index]                     */
+} arc_mismatch_t;
+
+typedef struct {
+    uint64_t n;             /* elements compared (global n when sharded)            */
+    uint64_t n_mismatch;    /* exact number of mismatches                           */
+    double max_abs_err;     /* max defined d; 0 for empty / all-NaN                 */
+    double max_rel_err;     /* max defined r; 0 for integer dtypes                  */
+    uint64_t n_reported;    /* = min(n_mismatch, max_report)                        */
+    arc_mismatch_t *report; /* CALLER-owned, capacity >= min(max_report, n) entries;
+                               host memory (pageable or pinned) or device memory on
+                               the library's device (then nothing crosses PCIe)     */
+} arc_verify_result_t;
+
+typedef struct {
+    int device;                 /* CUDA device ordinal                                    */
+    void *stream;               /* cudaStream_t to enqueue on; NULL = a library-owned
+                                   non-blocking stream (the caller orders its own work);
+                                   (void*)1 = cudaStreamLegacy, the legacy default stream */
+    int rank, nranks;           /* sharded mode when nranks > 1                           */
+    const void *nccl_unique_id; /* 128-byte ncclUniqueId (same on all ranks) if nranks > 1 */
+} arc_verify_opts_t;
+
+typedef struct {
+    const void *out;  /* region output computed by the GPU kernel                  */
+    const void *ref;  /* sequential reference output                               */
+    uint64_t n;       /* elements (row-major flattened)                            */
+    arc_dtype_t dtype;
+    double abs_tol, rel_tol;
+    uint64_t max_report;
+    const char *name; /* for printing only; may be NULL                            */
+} arc_verify_region_t;
+
+/*
+ * arc_verify_init -- create the process context.
+ *   opts == NULL: device 0, library-owned stream, one rank.
+ *   nranks > 1: sharded mode; nccl_unique_id must be the id produced by
+ *   arc_verify_get_unique_id on one rank and shared with all ranks; NCCL
+ *   (libnccl.so.2, the one already loaded by the process if any) is opened
+ *   at run time.
+ * Errors: ARC_E_INVAL (bad device / rank / nranks, missing id), ARC_E_CUDA,
+ * ARC_E_NCCL.  Calling init twice without finalize returns ARC_E_INVAL.
+ */
+int arc_verify_init(const arc_verify_opts_t *opts);
+
+/*
+ * arc_verify_compare -- verify one region: out[0..n) against ref[0..n).
+ *   out, ref : device pointers on the library's device, OR host pointers
+ *              (pinned or pageable); host inputs are streamed to the device in
+ *              chunks that overlap the comparison (the paper's data flow, where
+ *              the sequential reference lives in host memory).
+ *              Each pointer must be aligned to the element size.
+ *   n        : elements; n == 0 is legal (all-zero result).
+ *   dtype    : element type of both arrays.
+ *   abs_tol, rel_tol : finite and >= 0 (ignored for integer dtypes).
+ *   max_report : report capacity / truncation; 0 = count only.
+ *   result   : caller-owned; result->report must hold min(max_report, n)
+ *              entries when max_report > 0.
+ * Sharded mode (nranks > 1): COLLECTIVE -- every rank calls it with the same
+ * dtype, tolerances and max_report; out/ref/n are the rank's contiguous shard;
+ * global index = sum of n over lower ranks + local index; every rank receives
+ * the identical global result.
+ * Errors: ARC_E_INVAL (NULL arrays with n > 0, unknown dtype, NaN / negative /
+ * infinite tolerance, NULL result, NULL report with max_report > 0, misaligned
+ * pointer, device pointer on another device), ARC_E_NOINIT, ARC_E_CUDA,
+ * ARC_E_NCCL, ARC_E_NOMEM.
+ */
+int arc_verify_compare(const void *out, const void *ref, uint64_t n, arc_dtype_t dtype,
+                       double abs_tol, double rel_tol, uint64_t max_report,
+                       arc_verify_result_t *result);
+
+/*
+ * arc_verify_batch -- verify n_regions regions ("all data written by the kernels
+ * are examined") in ONE grid when all inputs are device-resident.
+ * results[k] equals what arc_verify_compare would return for regions[k] alone.
+ * Same argument rules as arc_verify_compare, per region.  Not collective: in
+ * sharded mode the batch is verified locally on each rank.
+ */
+int arc_verify_batch(const arc_verify_region_t *regions, size_t n_regions,
+                     arc_verify_result_t *results);
+
+/* Release the workspace, the NCCL communicator and the owned stream. */
+int arc_verify_finalize(void);
+
+/* Static text for a status code. */
+const char *arc_verify_strerror(int status);
+
+/* Text of the last failing CUDA/NCCL call in this process (static buffer). */
+const char *arc_verify_last_error(void);
+
+/* Enqueue subsequent work on `stream` (cudaStream_t on the library's device). */
+int arc_verify_set_stream(void *stream);
+
+/* Fill `id` (128 bytes) with a fresh ncclUniqueId for sharded init.
+ * Errors: ARC_E_NCCL if NCCL cannot be loaded. */
+int arc_verify_get_unique_id(void *id);
+
+/*
+ * Kernel timing for benchmarks: when enabled, the library records CUDA events
+ * on its stream around every compare-kernel launch and accumulates the launch
+ * count and total device time (ms) until arc_verify_kernel_stats(..., reset=1).
+ */
+int arc_verify_set_timing(int enable);
+int arc_verify_kernel_stats(uint64_t *launches, double *total_ms, int reset);
+
+/* ABI version (major << 16 | minor). */
+uint32_t arc_verify_version(void);
+
+/* ------------------------------------------------------------------------
+ * Sharded building blocks (the cross-GPU merge, DESIGN.md sec. 2 step a8).
+ * The paper is single-GPU; sharding one large output array across the
+ * GPUs of one box is this build's extension.  arc_verify_compare in sharded
+ * mode = arc_verify_shard_local -> ncclAllGather of the packets ->
+ * arc_verify_shard_merge (+ grouped ncclBroadcast of report entries that do
+ * not fit in a packet).  The pieces are exported so a single GPU can run the
+ * exact merge path over P simulated shards ("loopback"), and so host code can
+ * check the merge plan without a GPU.
+ * ------------------------------------------------------------------------ */
+
+/* Per-shard summary header, the first 32 bytes of a packet. */
+typedef struct {
+    uint64_t n;            /* shard length (elements)            */
+    uint64_t n_mismatch;   /* local exact count                  */
+    uint64_t max_abs_bits; /* bit pattern of the local max_abs   */
+    uint64_t max_rel_bits; /* bit pattern of the local max_rel   */
+} arc_shard_header_t;
+
+/* Where rank r's entries land in the global report. */
+typedef struct {
+    uint64_t index_offset; /* sum of n over lower ranks (global index base)          */
+    uint64_t prefix;       /* sum of n_mismatch over lower ranks (report position)   */
+    uint64_t contrib;      /* min(n_mismatch_r, max(0, max_report - prefix))         */
+} arc_shard_plan_t;
+
+/*
+ * arc_verify_merge_plan -- HOST function, needs no GPU and no init.  Given the
+ * nranks headers in rank order, fill plan[0..nranks) and the global header
+ * (sum of counts and n, max of the max bit patterns -- valid because the
+ * values are non-negative doubles).  Errors: ARC_E_INVAL on NULL pointers or
+ * nranks < 1.
+ */
+int arc_verify_merge_plan(const arc_shard_header_t *hdrs, int nranks, uint64_t max_report,
+                          arc_shard_plan_t *plan, arc_shard_header_t *global);
+
+/* Bytes of a packet holding `entries` report entries: 32 + 24 * entries. */
+size_t arc_verify_packet_bytes(uint64_t entries);
+
+/*
+ * arc_verify_shard_local -- compare one local shard (device pointers) and write
+ * its packet to packet_dev (device memory, capacity
+ * arc_verify_packet_bytes(max(packet_entries, min(max_report, n))) bytes):
+ * header, then the first min(n_mismatch, max_report) local mismatches with
+ * LOCAL indices.  Errors as arc_verify_compare.
+ */
+int arc_verify_shard_local(const void *out, const void *ref, uint64_t n, arc_dtype_t dtype, double abs_tol,
+                           double rel_tol, uint64_t max_report, void *packet_dev, uint64_t packet_entries);
+
+/*
+ * arc_verify_shard_merge -- merge nranks gathered packets (device memory,
+ * rank r's packet at byte offset r * arc_verify_packet_bytes(packet_entries))
+ * into the global result, on the GPU.  result->report as in
+ * arc_verify_compare.  Every contribution must fit in its packet
+ * (plan.contrib <= packet_entries), else ARC_E_UNSUPPORTED (the collective
+ * path then broadcasts the remainder).
+ */
+int arc_verify_shard_merge(const void *gathered_dev, int nranks, uint64_t packet_entries, uint64_t max_report,
+                           arc_verify_result_t *result);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ARC_VERIFY_H */

@@ -1,0 +1,331 @@
+"""paper_conf_ipps_leelv14_b200 -- B200-native kernel-verification result comparison.
+
+Thin ctypes binding over ``libarcverify.so`` (C ABI: include/arc_verify.h).
+The functions named ``arc_verify_*`` mirror the C entry points one to one and
+only marshal arguments; every step of the comparison runs in the library's
+CUDA kernels.  ``compare`` / ``batch`` are conveniences over torch tensors
+(PyTorch is used for device memory, streams and process groups only).
+
+There is no CPU fallback: importing this package without the built library
+raises ImportError.  Build it with ``python -m paper_conf_ipps_leelv14_b200._build``
+or ``__graft_entry__.build()``.
+
+Paper: S. Lee, D. Li, J. S. Vetter, "Interactive Program Debugging and
+Optimization for Directive-Based, Efficient GPU Computing", IPDPS 2014,
+sec. III-A: verify each GPU kernel's outputs against the
+sequential CPU outputs under a user-configurable error margin and report the
+differences.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass, field
+from typing import Optional, Sequence
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libarcverify.so")
+
+ARC_OK, ARC_E_INVAL, ARC_E_NOINIT, ARC_E_CUDA, ARC_E_NCCL, ARC_E_NOMEM, ARC_E_UNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
+ARC_F32, ARC_F64, ARC_I32, ARC_I64, ARC_U8 = 0, 1, 2, 3, 4
+DTYPE_CODES = {"f32": ARC_F32, "f64": ARC_F64, "i32": ARC_I32, "i64": ARC_I64, "u8": ARC_U8}
+
+EXPORTED = [
+    "arc_verify_init", "arc_verify_compare", "arc_verify_batch", "arc_verify_finalize",
+    "arc_verify_strerror", "arc_verify_last_error", "arc_verify_set_stream",
+    "arc_verify_get_unique_id", "arc_verify_set_timing", "arc_verify_kernel_stats",
+    "arc_verify_version", "arc_verify_merge_plan", "arc_verify_packet_bytes",
+    "arc_verify_shard_local", "arc_verify_shard_merge",
+]
+
+
+class arc_mismatch_t(ctypes.Structure):
+    _fields_ = [("index", ctypes.c_uint64), ("out_bits", ctypes.c_uint64), ("ref_bits", ctypes.c_uint64)]
+
+
+class arc_verify_result_t(ctypes.Structure):
+    _fields_ = [
+        ("n", ctypes.c_uint64), ("n_mismatch", ctypes.c_uint64),
+        ("max_abs_err", ctypes.c_double), ("max_rel_err", ctypes.c_double),
+        ("n_reported", ctypes.c_uint64), ("report", ctypes.c_void_p),
+    ]
+
+
+class arc_verify_opts_t(ctypes.Structure):
+    _fields_ = [("device", ctypes.c_int), ("stream", ctypes.c_void_p), ("rank", ctypes.c_int),
+                ("nranks", ctypes.c_int), ("nccl_unique_id", ctypes.c_void_p)]
+
+
+class arc_verify_region_t(ctypes.Structure):
+    _fields_ = [("out", ctypes.c_void_p), ("ref", ctypes.c_void_p), ("n", ctypes.c_uint64),
+                ("dtype", ctypes.c_int), ("abs_tol", ctypes.c_double), ("rel_tol", ctypes.c_double),
+                ("max_report", ctypes.c_uint64), ("name", ctypes.c_char_p)]
+
+
+class arc_shard_header_t(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_uint64), ("n_mismatch", ctypes.c_uint64),
+                ("max_abs_bits", ctypes.c_uint64), ("max_rel_bits", ctypes.c_uint64)]
+
+
+class arc_shard_plan_t(ctypes.Structure):
+    _fields_ = [("index_offset", ctypes.c_uint64), ("prefix", ctypes.c_uint64), ("contrib", ctypes.c_uint64)]
+
+
+CUDA_STREAM_LEGACY = 1  # cudaStreamLegacy
+
+REPORT_DTYPE = np.dtype([("index", "<u8"), ("out_bits", "<u8"), ("ref_bits", "<u8")])
+
+
+def _load() -> ctypes.CDLL:
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: build it with __graft_entry__.build() "
+                          "(there is no CPU fallback)")
+    lib = ctypes.CDLL(LIB_PATH)
+    P, U64, I, D, SZ = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int, ctypes.c_double, ctypes.c_size_t
+    sig = {
+        "arc_verify_init": (I, [ctypes.POINTER(arc_verify_opts_t)]),
+        "arc_verify_compare": (I, [P, P, U64, I, D, D, U64, ctypes.POINTER(arc_verify_result_t)]),
+        "arc_verify_batch": (I, [ctypes.POINTER(arc_verify_region_t), SZ, ctypes.POINTER(arc_verify_result_t)]),
+        "arc_verify_finalize": (I, []),
+        "arc_verify_strerror": (ctypes.c_char_p, [I]),
+        "arc_verify_last_error": (ctypes.c_char_p, []),
+        "arc_verify_set_stream": (I, [P]),
+        "arc_verify_get_unique_id": (I, [P]),
+        "arc_verify_set_timing": (I, [I]),
+        "arc_verify_kernel_stats": (I, [ctypes.POINTER(U64), ctypes.POINTER(D), I]),
+        "arc_verify_version": (ctypes.c_uint32, []),
+        "arc_verify_merge_plan": (I, [ctypes.POINTER(arc_shard_header_t), I, U64,
+                                      ctypes.POINTER(arc_shard_plan_t), ctypes.POINTER(arc_shard_header_t)]),
+        "arc_verify_packet_bytes": (SZ, [U64]),
+        "arc_verify_shard_local": (I, [P, P, U64, I, D, D, U64, P, U64]),
+        "arc_verify_shard_merge": (I, [P, I, U64, U64, ctypes.POINTER(arc_verify_result_t)]),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(lib, name)
+        f.restype, f.argtypes = res, args
+    return lib
+
+
+_lib = _load()
+
+
+class ArcVerifyError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        self.status = status
+        msg = _lib.arc_verify_strerror(status).decode()
+        detail = _lib.arc_verify_last_error().decode()
+        super().__init__(f"{where}: {msg} ({status}){': ' + detail if detail else ''}")
+
+
+def _check(status: int, where: str) -> None:
+    if status != ARC_OK:
+        raise ArcVerifyError(status, where)
+
+
+# --------------------------------------------------------- raw C entry points
+def arc_verify_init(device: int = 0, stream: Optional[int] = None, rank: int = 0, nranks: int = 1,
+                    nccl_unique_id: Optional[bytes] = None) -> None:
+    opts = arc_verify_opts_t(device, stream or None, rank, nranks, None)
+    buf = None
+    if nccl_unique_id is not None:
+        buf = ctypes.create_string_buffer(bytes(nccl_unique_id), 128)
+        opts.nccl_unique_id = ctypes.cast(buf, ctypes.c_void_p)
+    _check(_lib.arc_verify_init(ctypes.byref(opts)), "arc_verify_init")
+
+
+def arc_verify_finalize() -> None:
+    _check(_lib.arc_verify_finalize(), "arc_verify_finalize")
+
+
+def arc_verify_compare(out_ptr: int, ref_ptr: int, n: int, dtype: int, abs_tol: float, rel_tol: float,
+                       max_report: int, result: arc_verify_result_t) -> None:
+    _check(_lib.arc_verify_compare(out_ptr or None, ref_ptr or None, n, dtype, abs_tol, rel_tol, max_report,
+                                   ctypes.byref(result)), "arc_verify_compare")
+
+
+def arc_verify_batch(regions, results) -> None:
+    n = len(regions)
+    _check(_lib.arc_verify_batch(regions, n, results), "arc_verify_batch")
+
+
+def arc_verify_set_stream(stream: int) -> None:
+    _check(_lib.arc_verify_set_stream(stream), "arc_verify_set_stream")
+
+
+def arc_verify_get_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(_lib.arc_verify_get_unique_id(buf), "arc_verify_get_unique_id")
+    return buf.raw
+
+
+def arc_verify_set_timing(enable: bool) -> None:
+    _check(_lib.arc_verify_set_timing(int(enable)), "arc_verify_set_timing")
+
+
+def arc_verify_kernel_stats(reset: bool = False) -> tuple[int, float]:
+    n, ms = ctypes.c_uint64(), ctypes.c_double()
+    _check(_lib.arc_verify_kernel_stats(ctypes.byref(n), ctypes.byref(ms), int(reset)), "arc_verify_kernel_stats")
+    return int(n.value), float(ms.value)
+
+
+def arc_verify_version() -> int:
+    return int(_lib.arc_verify_version())
+
+
+def arc_verify_packet_bytes(entries: int) -> int:
+    return int(_lib.arc_verify_packet_bytes(entries))
+
+
+def arc_verify_merge_plan(headers: Sequence[tuple], max_report: int):
+    """headers: [(n, n_mismatch, max_abs_bits, max_rel_bits)] in rank order (host only)."""
+    p = len(headers)
+    H = (arc_shard_header_t * p)(*[arc_shard_header_t(*h) for h in headers])
+    plan = (arc_shard_plan_t * p)()
+    g = arc_shard_header_t()
+    _check(_lib.arc_verify_merge_plan(H, p, max_report, plan, ctypes.byref(g)), "arc_verify_merge_plan")
+    return ([(x.index_offset, x.prefix, x.contrib) for x in plan],
+            (g.n, g.n_mismatch, g.max_abs_bits, g.max_rel_bits))
+
+
+def arc_verify_shard_local(out_ptr, ref_ptr, n, dtype, abs_tol, rel_tol, max_report, packet_ptr, packet_entries):
+    _check(_lib.arc_verify_shard_local(out_ptr or None, ref_ptr or None, n, dtype, abs_tol, rel_tol, max_report,
+                                       packet_ptr, packet_entries), "arc_verify_shard_local")
+
+
+def arc_verify_shard_merge(gathered_ptr, nranks, packet_entries, max_report, result: arc_verify_result_t):
+    _check(_lib.arc_verify_shard_merge(gathered_ptr, nranks, packet_entries, max_report, ctypes.byref(result)),
+           "arc_verify_shard_merge")
+
+
+# ------------------------------------------------------------- conveniences
+@dataclass
+class Result:
+    n: int
+    n_mismatch: int
+    max_abs_err: float
+    max_rel_err: float
+    n_reported: int
+    report: np.ndarray = field(repr=False)  # REPORT_DTYPE (host), or a device tensor view
+
+
+_TORCH_CODES = None
+
+
+def dtype_code(t) -> int:
+    global _TORCH_CODES
+    import torch
+
+    if _TORCH_CODES is None:
+        _TORCH_CODES = {torch.float32: ARC_F32, torch.float64: ARC_F64, torch.int32: ARC_I32,
+                        torch.int64: ARC_I64, torch.uint8: ARC_U8}
+    try:
+        return _TORCH_CODES[t.dtype]
+    except KeyError:
+        raise TypeError(f"unsupported dtype {t.dtype}") from None
+
+
+_state = {"init": False}
+
+
+def init(device: Optional[int] = None, stream=None, rank: int = 0, nranks: int = 1,
+         nccl_unique_id: Optional[bytes] = None) -> None:
+    """Initialise on ``device`` enqueuing on ``stream`` (default: torch's current stream)."""
+    import torch
+
+    if device is None:
+        device = torch.cuda.current_device()
+    if stream is None:
+        stream = torch.cuda.current_stream(device)
+    handle = stream.cuda_stream if hasattr(stream, "cuda_stream") else stream
+    if not handle:
+        handle = CUDA_STREAM_LEGACY  # torch's default stream is the legacy NULL stream
+    arc_verify_init(device, handle, rank, nranks, nccl_unique_id)
+    _state["init"] = True
+
+
+def init_distributed(group=None) -> None:
+    """Sharded init over a torch.distributed group: rank 0 creates the NCCL id."""
+    import torch
+    import torch.distributed as dist
+
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    obj = [arc_verify_get_unique_id() if rank == 0 else None]
+    dist.broadcast_object_list(obj, src=0, group=group)
+    init(torch.cuda.current_device(), None, rank, world, obj[0])
+
+
+def finalize() -> None:
+    if _state["init"]:
+        arc_verify_finalize()
+        _state["init"] = False
+
+
+def _report_buffer(cap: int):
+    arr = np.zeros(max(cap, 1), dtype=REPORT_DTYPE)
+    return arr, arr.ctypes.data
+
+
+def compare(out, ref, abs_tol: float = 0.0, rel_tol: float = 0.0, max_report: int = 1 << 20,
+            report=None, n: Optional[int] = None) -> Result:
+    """Verify ``out`` against ``ref`` (torch tensors, contiguous, same dtype).
+
+    Tensors may live on the library's CUDA device or in (pinned) host memory.
+    ``report``: optional preallocated buffer -- a numpy REPORT_DTYPE array or a
+    CUDA uint8/int64 tensor of >= 24*cap bytes (then the report stays on the GPU).
+    """
+    if out.dtype != ref.dtype:
+        raise TypeError("out and ref dtypes differ")
+    if not (out.is_contiguous() and ref.is_contiguous()):
+        raise ValueError("tensors must be contiguous")
+    if n is None:
+        n = out.numel()
+        if ref.numel() != n:
+            raise ValueError("size mismatch")
+    cap = min(int(max_report), n)
+    if report is None:
+        rep_arr, rep_ptr = _report_buffer(cap)
+    elif isinstance(report, np.ndarray):
+        rep_arr, rep_ptr = report, report.ctypes.data
+    else:
+        rep_arr, rep_ptr = report, report.data_ptr()
+    res = arc_verify_result_t()
+    res.report = rep_ptr if max_report > 0 else None
+    arc_verify_compare(out.data_ptr() if n else 0, ref.data_ptr() if n else 0, n, dtype_code(out),
+                       float(abs_tol), float(rel_tol), int(max_report), res)
+    if isinstance(rep_arr, np.ndarray):
+        rep = rep_arr[: res.n_reported]
+    else:
+        rep = rep_arr
+    return Result(int(res.n), int(res.n_mismatch), float(res.max_abs_err), float(res.max_rel_err),
+                  int(res.n_reported), rep)
+
+
+def batch(regions) -> list[Result]:
+    """regions: iterable of (out, ref, abs_tol, rel_tol, max_report[, name]) torch tensors."""
+    regions = list(regions)
+    R = len(regions)
+    regs = (arc_verify_region_t * R)()
+    results = (arc_verify_result_t * R)()
+    keep = []
+    for k, reg in enumerate(regions):
+        out, ref, at, rt, mr = reg[:5]
+        name = reg[5] if len(reg) > 5 else None
+        n = out.numel()
+        if ref.numel() != n or out.dtype != ref.dtype:
+            raise ValueError(f"region {k}: size/dtype mismatch")
+        arr, ptr = _report_buffer(min(int(mr), n))
+        keep.append(arr)
+        nm = name.encode() if name else None
+        keep.append(nm)
+        regs[k] = arc_verify_region_t(out.data_ptr() if n else None, ref.data_ptr() if n else None, n,
+                                      dtype_code(out), float(at), float(rt), int(mr), nm)
+        results[k].report = ptr if mr > 0 else None
+    arc_verify_batch(regs, results)
+    outs = []
+    for k in range(R):
+        r = results[k]
+        outs.append(Result(int(r.n), int(r.n_mismatch), float(r.max_abs_err), float(r.max_rel_err),
+                           int(r.n_reported), keep[2 * k][: r.n_reported]))
+    return outs

@@ -1,0 +1,595 @@
+// arcv_host.cu -- C ABI of include/arc_verify.h: context, workspace, launch
+// planning, host-input streaming, result materialisation.
+//
+// Steps of the hot path: a1 validation + dispatch happens
+// here; a2-a5 run in arcv_compare_kernel (arcv_device.cuh); a6 (summary and
+// report to the host) and a7 (one grid over many regions) are planned here; a8
+// (cross-GPU merge) lives in arcv_shard.cu.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <vector>
+
+#include "arc_verify.h"
+#include "arcv_device.cuh"
+#include "arcv_internal.h"
+
+namespace arcv {
+
+static char g_err[512] = "";
+
+void set_error(const char *fmt, ...) {
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+}
+
+int cuda_fail(cudaError_t e, const char *what) {
+    set_error("%s: %s", what, cudaGetErrorString(e));
+    return ARC_E_CUDA;
+}
+
+#define CK(call)                                                 \
+    do {                                                         \
+        cudaError_t e_ = (call);                                 \
+        if (e_ != cudaSuccess) return cuda_fail(e_, #call);      \
+    } while (0)
+
+Ctx *g_ctx = nullptr;
+
+// ------------------------------------------------------------------ kernels
+typedef void (*KernelFn)(Params);
+static KernelFn kernel_for_stages(int s) {
+    switch (s) {
+        case 2: return arcv_compare_kernel<2>;
+        case 4: return arcv_compare_kernel<4>;
+        case 6: return arcv_compare_kernel<6>;
+        default: return arcv_compare_kernel<3>;
+    }
+}
+
+static int env_int(const char *name, int dflt) {
+    const char *v = getenv(name);
+    return v && *v ? atoi(v) : dflt;
+}
+
+// ---------------------------------------------------------- device buffers
+template <typename T>
+static int grow_device(T **p, size_t *cap, size_t need, bool zero, cudaStream_t st) {
+    if (need <= *cap) return ARC_OK;
+    size_t ncap = std::max(need, *cap * 2);
+    if (*p) {
+        CK(cudaStreamSynchronize(st));
+        CK(cudaFree(*p));
+        *p = nullptr;
+        *cap = 0;
+    }
+    cudaError_t e = cudaMalloc(reinterpret_cast<void **>(p), ncap * sizeof(T));
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        set_error("cudaMalloc(%zu bytes) failed: %s", ncap * sizeof(T), cudaGetErrorString(e));
+        return ARC_E_NOMEM;
+    }
+    if (zero) CK(cudaMemsetAsync(*p, 0, ncap * sizeof(T), st));
+    *cap = ncap;
+    return ARC_OK;
+}
+
+template <typename T>
+static int grow_pinned(T **p, size_t *cap, size_t need) {
+    if (need <= *cap) return ARC_OK;
+    size_t ncap = std::max(need, *cap * 2);
+    if (*p) CK(cudaFreeHost(*p));
+    *p = nullptr;
+    *cap = 0;
+    cudaError_t e = cudaMallocHost(reinterpret_cast<void **>(p), ncap * sizeof(T));
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        set_error("cudaMallocHost(%zu bytes) failed: %s", ncap * sizeof(T), cudaGetErrorString(e));
+        return ARC_E_NOMEM;
+    }
+    *cap = ncap;
+    return ARC_OK;
+}
+
+PtrKind classify(const void *p, int device) {
+    cudaPointerAttributes a;
+    cudaError_t e = cudaPointerGetAttributes(&a, p);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return PK_HOST;
+    }
+    switch (a.type) {
+        case cudaMemoryTypeDevice: return a.device == device ? PK_DEVICE : PK_BAD;
+        case cudaMemoryTypeManaged: return PK_DEVICE;
+        default: return PK_HOST;  // pinned (cudaMemoryTypeHost) or pageable
+    }
+}
+
+int validate_region(const void *out, const void *ref, uint64_t n, int dtype, double abs_tol, double rel_tol,
+                    uint64_t max_report, const arc_verify_result_t *res) {
+    if (!res) { set_error("result is NULL"); return ARC_E_INVAL; }
+    if (dtype < ARC_F32 || dtype > ARC_U8) { set_error("unknown dtype %d", dtype); return ARC_E_INVAL; }
+    if (!(abs_tol >= 0.0) || !(rel_tol >= 0.0) || std::isinf(abs_tol) || std::isinf(rel_tol)) {
+        set_error("tolerances must be finite and >= 0 (abs_tol=%g rel_tol=%g)", abs_tol, rel_tol);
+        return ARC_E_INVAL;
+    }
+    if (n > 0 && (!out || !ref)) { set_error("NULL array with n > 0"); return ARC_E_INVAL; }
+    if (max_report > 0 && !res->report) { set_error("report is NULL with max_report > 0"); return ARC_E_INVAL; }
+    const uintptr_t es = elem_size((uint32_t)dtype);
+    if (n > 0 && (((uintptr_t)out % es) || ((uintptr_t)ref % es))) {
+        set_error("array pointer not aligned to the element size");
+        return ARC_E_INVAL;
+    }
+    return ARC_OK;
+}
+
+// ------------------------------------------------------------------ launch
+int launch_segments(Ctx &c, const Seg *segs, uint32_t n_segs, uint64_t total_tiles, uint32_t acc_lo,
+                    uint32_t n_acc, bool finalize) {
+    Params p;
+    memset(&p, 0, sizeof(p));
+    if (n_segs <= (uint32_t)kMaxInlineSegs) {
+        memcpy(p.inline_segs, segs, n_segs * sizeof(Seg));
+        p.segs = nullptr;
+    } else {
+        int st = grow_device(&c.seg_dev, &c.seg_dev_cap, n_segs, false, c.stream);
+        if (st) return st;
+        st = grow_pinned(&c.seg_host, &c.seg_host_cap, n_segs);
+        if (st) return st;
+        CK(cudaStreamSynchronize(c.stream));  // seg_host may still feed an earlier copy
+        memcpy(c.seg_host, segs, n_segs * sizeof(Seg));
+        CK(cudaMemcpyAsync(c.seg_dev, c.seg_host, n_segs * sizeof(Seg), cudaMemcpyHostToDevice, c.stream));
+        p.segs = c.seg_dev;
+    }
+    p.n_segs = n_segs;
+    p.n_acc = n_acc;
+    p.total_tiles = total_tiles;
+    p.ticket = c.counters;
+    p.ticket_base = c.ticket_base;
+    p.done = c.counters + 1;
+    p.done_base = c.done_base;
+    p.status = c.status;
+    p.epoch_tag = (uint64_t)c.epoch << kEpochShift;
+    p.acc = c.acc + acc_lo;
+    p.result = c.result_dev + acc_lo;
+    p.finalize = finalize ? 1 : 0;
+    p.flags = (uint32_t)c.flags;
+
+    const uint64_t max_grid = (uint64_t)c.num_sms * (uint64_t)c.ctas_per_sm;
+    const uint32_t grid = (uint32_t)std::min<uint64_t>(total_tiles, max_grid);
+    const size_t smem = (size_t)c.stages * kStageBytes;
+    const bool timed = c.timing && c.n_ev < Ctx::kMaxEv;
+    if (timed) CK(cudaEventRecord(c.ev[c.n_ev][0], c.stream));
+    kernel_for_stages(c.stages)<<<grid, kThreads, smem, c.stream>>>(p);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "arcv_compare_kernel launch");
+    if (timed) {
+        CK(cudaEventRecord(c.ev[c.n_ev][1], c.stream));
+        c.n_ev++;
+    }
+    c.launches++;
+    c.ticket_base += total_tiles + grid;
+    if (finalize) c.done_base += grid;
+    return ARC_OK;
+}
+
+static int collect_timing(Ctx &c) {
+    for (int i = 0; i < c.n_ev; ++i) {
+        float ms = 0.f;
+        CK(cudaEventElapsedTime(&ms, c.ev[i][0], c.ev[i][1]));
+        c.timed_ms += ms;
+        c.timed_launches++;
+    }
+    c.n_ev = 0;
+    return ARC_OK;
+}
+
+static uint64_t tiles_of(uint64_t n, uint32_t dtype) {
+    const uint64_t te = kTileBytes / elem_size(dtype);
+    return (n + te - 1) / te;
+}
+
+// Prepare per-call state: epoch, workspace sizes.
+static int begin_call(Ctx &c, uint64_t status_slots, uint32_t n_acc) {
+    int st = grow_device(&c.status, &c.status_cap, std::max<uint64_t>(status_slots, 1), true, c.stream);
+    if (st) return st;
+    st = grow_device(&c.acc, &c.acc_cap, std::max<uint32_t>(n_acc, 1), true, c.stream);
+    if (st) return st;
+    st = grow_device(&c.result_dev, &c.result_dev_cap, std::max<uint32_t>(n_acc, 1), false, c.stream);
+    if (st) return st;
+    st = grow_pinned(&c.result_host, &c.result_host_cap, std::max<uint32_t>(n_acc, 1));
+    if (st) return st;
+    c.epoch = (uint16_t)(c.epoch + 1);
+    if (c.epoch == 0) {  // wrapped: stale words could alias the new epoch
+        CK(cudaMemsetAsync(c.status, 0, c.status_cap * sizeof(uint64_t), c.stream));
+        c.epoch = 1;
+    }
+    return ARC_OK;
+}
+
+// Stream one region whose out and/or ref live in host memory through the chunk
+// ring: H2D copies on the copy stream overlap the compare of the previous chunk.
+static int stream_region(Ctx &c, const void *out, const void *ref, bool out_dev, bool ref_dev, uint64_t n,
+                         uint32_t dtype, double at, double rt, uint64_t max_report, arc_mismatch_t *report,
+                         uint64_t status_base, uint32_t slot) {
+    const uint64_t es = elem_size(dtype);
+    const uint64_t te = kTileBytes / es;
+    const uint64_t chunk_elems = std::max<uint64_t>(te, (Ctx::kChunkBytes / es) / te * te);
+    if (!c.chunk_buf[0][0]) {
+        for (int b = 0; b < Ctx::kNBuf; ++b)
+            for (int s = 0; s < 2; ++s) {
+                cudaError_t e = cudaMalloc(&c.chunk_buf[b][s], Ctx::kChunkBytes);
+                if (e != cudaSuccess) {
+                    cudaGetLastError();
+                    set_error("cudaMalloc(chunk buffer) failed: %s", cudaGetErrorString(e));
+                    return ARC_E_NOMEM;
+                }
+            }
+    }
+    const uint64_t nchunks = (n + chunk_elems - 1) / chunk_elems;
+    for (uint64_t ci = 0; ci < nchunks; ++ci) {
+        const int b = (int)(ci % Ctx::kNBuf);
+        const uint64_t e0 = ci * chunk_elems;
+        const uint64_t ne = std::min(chunk_elems, n - e0);
+        CK(cudaStreamWaitEvent(c.copy_stream, c.ev_free[b], 0));
+        const uint8_t *po = static_cast<const uint8_t *>(out) + e0 * es;
+        const uint8_t *pr = static_cast<const uint8_t *>(ref) + e0 * es;
+        if (!out_dev) {
+            CK(cudaMemcpyAsync(c.chunk_buf[b][0], po, ne * es, cudaMemcpyHostToDevice, c.copy_stream));
+            po = static_cast<const uint8_t *>(c.chunk_buf[b][0]);
+        }
+        if (!ref_dev) {
+            CK(cudaMemcpyAsync(c.chunk_buf[b][1], pr, ne * es, cudaMemcpyHostToDevice, c.copy_stream));
+            pr = static_cast<const uint8_t *>(c.chunk_buf[b][1]);
+        }
+        c.h2d_bytes += (out_dev ? 0 : ne * es) + (ref_dev ? 0 : ne * es);
+        CK(cudaEventRecord(c.ev_copy[b], c.copy_stream));
+        CK(cudaStreamWaitEvent(c.stream, c.ev_copy[b], 0));
+        Seg g;
+        memset(&g, 0, sizeof(g));
+        g.out = po;
+        g.ref = pr;
+        g.n = ne;
+        g.tile_begin = 0;
+        g.status_begin = status_base + e0 / te;
+        g.chain_begin = status_base;
+        g.index_base = e0;
+        g.abs_tol = at;
+        g.rel_tol = rt;
+        g.max_report = max_report;
+        g.report = report;
+        g.acc_slot = 0;
+        g.dtype = dtype;
+        int st = launch_segments(c, &g, 1, tiles_of(ne, dtype), slot, 1, ci + 1 == nchunks);
+        if (st) return st;
+        CK(cudaEventRecord(c.ev_free[b], c.stream));
+    }
+    return ARC_OK;
+}
+
+// Local (single-GPU) verification of R regions.  Results go to results[k]; a
+// region's report goes to its device report pointer, or to the device staging
+// buffer and then to host memory.  When `dev_reports` is non-NULL the caller
+// supplies the device report target per region instead (sharded packets).
+int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_result_t *results,
+              arc_mismatch_t *const *dev_reports, bool d2h_reports, Acc *summaries_out) {
+    struct Plan {
+        bool out_dev, ref_dev, stream;
+        arc_mismatch_t *dreport;  // device target
+        bool host_report;
+        uint64_t stage_off;
+        uint64_t tiles, status_base;
+    };
+    std::vector<Plan> plan(R);
+    uint64_t status_slots = 0, stage_entries = 0;
+    for (size_t k = 0; k < R; ++k) {
+        const arc_verify_region_t &r = regs[k];
+        int st = validate_region(r.out, r.ref, r.n, r.dtype, r.abs_tol, r.rel_tol, r.max_report, &results[k]);
+        if (st) return st;
+        Plan &pl = plan[k];
+        pl.out_dev = pl.ref_dev = true;
+        if (r.n > 0) {
+            const PtrKind ko = classify(r.out, c.device), kr = classify(r.ref, c.device);
+            if (ko == PK_BAD || kr == PK_BAD) {
+                set_error("region %zu: device pointer belongs to another device", k);
+                return ARC_E_INVAL;
+            }
+            pl.out_dev = ko == PK_DEVICE;
+            pl.ref_dev = kr == PK_DEVICE;
+        }
+        pl.stream = !(pl.out_dev && pl.ref_dev);
+        pl.tiles = tiles_of(r.n, r.dtype);
+        pl.status_base = status_slots;
+        status_slots += pl.tiles;
+        const uint64_t cap = std::min<uint64_t>(r.max_report, r.n);
+        pl.host_report = false;
+        pl.dreport = nullptr;
+        if (cap > 0) {
+            if (dev_reports) {
+                pl.dreport = dev_reports[k];
+            } else if (classify(results[k].report, c.device) == PK_DEVICE) {
+                pl.dreport = results[k].report;
+            } else {
+                pl.host_report = true;
+                pl.stage_off = stage_entries;
+                stage_entries += cap;
+            }
+        }
+    }
+    int st = begin_call(c, status_slots, (uint32_t)R);
+    if (st) return st;
+    if (stage_entries) {
+        st = grow_device(&c.report_stage, &c.report_stage_cap, stage_entries, false, c.stream);
+        if (st) return st;
+    }
+    for (size_t k = 0; k < R; ++k)
+        if (plan[k].host_report) plan[k].dreport = c.report_stage + plan[k].stage_off;
+
+    // One grid over every device-resident region (a7).
+    std::vector<Seg> segs;
+    std::vector<uint32_t> dev_regions;
+    uint64_t tiles = 0;
+    for (size_t k = 0; k < R; ++k) {
+        const arc_verify_region_t &r = regs[k];
+        if (plan[k].stream || r.n == 0) continue;
+        dev_regions.push_back((uint32_t)k);
+    }
+    // accumulator slots: device regions occupy [0, D) in region order
+    std::vector<uint32_t> slot_of(R, 0);
+    uint32_t next_slot = 0;
+    for (uint32_t k : dev_regions) slot_of[k] = next_slot++;
+    const uint32_t n_dev_slots = next_slot;
+    for (size_t k = 0; k < R; ++k)
+        if (plan[k].stream && regs[k].n > 0) slot_of[k] = next_slot++;
+    for (uint32_t k : dev_regions) {
+        const arc_verify_region_t &r = regs[k];
+        Seg g;
+        memset(&g, 0, sizeof(g));
+        g.out = static_cast<const uint8_t *>(r.out);
+        g.ref = static_cast<const uint8_t *>(r.ref);
+        g.n = r.n;
+        g.tile_begin = tiles;
+        g.status_begin = plan[k].status_base;
+        g.chain_begin = plan[k].status_base;
+        g.index_base = 0;
+        g.abs_tol = r.abs_tol;
+        g.rel_tol = r.rel_tol;
+        g.max_report = plan[k].dreport ? r.max_report : 0;
+        g.report = plan[k].dreport;
+        g.acc_slot = slot_of[k];
+        g.dtype = (uint32_t)r.dtype;
+        segs.push_back(g);
+        tiles += plan[k].tiles;
+    }
+    if (!segs.empty()) {
+        st = launch_segments(c, segs.data(), (uint32_t)segs.size(), tiles, 0, n_dev_slots, true);
+        if (st) return st;
+    }
+    for (size_t k = 0; k < R; ++k) {
+        const arc_verify_region_t &r = regs[k];
+        if (!plan[k].stream || r.n == 0) continue;
+        st = stream_region(c, r.out, r.ref, plan[k].out_dev, plan[k].ref_dev, r.n, (uint32_t)r.dtype, r.abs_tol,
+                           r.rel_tol, plan[k].dreport ? r.max_report : 0, plan[k].dreport, plan[k].status_base,
+                           slot_of[k]);
+        if (st) return st;
+    }
+    const uint32_t n_slots = next_slot;
+    if (n_slots) {
+        CK(cudaMemcpyAsync(c.result_host, c.result_dev, n_slots * sizeof(Acc), cudaMemcpyDeviceToHost, c.stream));
+        CK(cudaStreamSynchronize(c.stream));
+    }
+    if (c.timing) {
+        st = collect_timing(c);
+        if (st) return st;
+    }
+    for (size_t k = 0; k < R; ++k) {
+        const arc_verify_region_t &r = regs[k];
+        Acc a;
+        memset(&a, 0, sizeof(a));
+        if (r.n > 0) a = c.result_host[slot_of[k]];
+        if (summaries_out) summaries_out[k] = a;
+        arc_verify_result_t &o = results[k];
+        o.n = r.n;
+        o.n_mismatch = a.count;
+        double ma, mr;
+        memcpy(&ma, &a.max_abs_bits, 8);
+        memcpy(&mr, &a.max_rel_bits, 8);
+        o.max_abs_err = ma;
+        o.max_rel_err = mr;
+        o.n_reported = std::min<uint64_t>(a.count, r.max_report);
+    }
+    if (d2h_reports) {
+        bool any = false;
+        for (size_t k = 0; k < R; ++k) {
+            if (!plan[k].host_report || results[k].n_reported == 0) continue;
+            CK(cudaMemcpyAsync(results[k].report, plan[k].dreport, results[k].n_reported * sizeof(arc_mismatch_t),
+                               cudaMemcpyDeviceToHost, c.stream));
+            any = true;
+        }
+        if (any) CK(cudaStreamSynchronize(c.stream));
+    }
+    return ARC_OK;
+}
+
+}  // namespace arcv
+
+using namespace arcv;
+
+// ====================================================================== C ABI
+extern "C" {
+
+uint32_t arc_verify_version(void) { return (1u << 16) | 0u; }
+
+const char *arc_verify_strerror(int status) {
+    switch (status) {
+        case ARC_OK: return "ok";
+        case ARC_E_INVAL: return "invalid argument";
+        case ARC_E_NOINIT: return "arc_verify_init has not been called";
+        case ARC_E_CUDA: return "CUDA runtime error";
+        case ARC_E_NCCL: return "NCCL error";
+        case ARC_E_NOMEM: return "out of memory";
+        case ARC_E_UNSUPPORTED: return "unsupported request";
+        default: return "unknown status";
+    }
+}
+
+const char *arc_verify_last_error(void) { return g_err; }
+
+int arc_verify_init(const arc_verify_opts_t *opts) {
+    if (g_ctx) { set_error("already initialised"); return ARC_E_INVAL; }
+    arc_verify_opts_t o;
+    memset(&o, 0, sizeof(o));
+    o.nranks = 1;
+    if (opts) o = *opts;
+    if (o.nranks < 1 || o.rank < 0 || o.rank >= o.nranks) { set_error("bad rank/nranks"); return ARC_E_INVAL; }
+    if (o.nranks > 1 && !o.nccl_unique_id) { set_error("nranks > 1 needs nccl_unique_id"); return ARC_E_INVAL; }
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess) { cudaGetLastError(); return cuda_fail(e, "cudaGetDeviceCount"); }
+    if (o.device < 0 || o.device >= ndev) { set_error("bad device %d (of %d)", o.device, ndev); return ARC_E_INVAL; }
+    CK(cudaSetDevice(o.device));
+    cudaDeviceProp prop;
+    CK(cudaGetDeviceProperties(&prop, o.device));
+    if (prop.major < 10) {
+        set_error("device %d is sm_%d%d; this build targets sm_100a", o.device, prop.major, prop.minor);
+        return ARC_E_UNSUPPORTED;
+    }
+    Ctx *c = new Ctx();
+    c->device = o.device;
+    c->rank = o.rank;
+    c->nranks = o.nranks;
+    c->num_sms = prop.multiProcessorCount;
+    if (o.stream) {
+        c->stream = static_cast<cudaStream_t>(o.stream);
+        c->own_stream = false;
+    } else {
+        CK(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking));
+        c->own_stream = true;
+    }
+    CK(cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking));
+    for (int b = 0; b < Ctx::kNBuf; ++b) {
+        CK(cudaEventCreateWithFlags(&c->ev_copy[b], cudaEventDisableTiming));
+        CK(cudaEventCreateWithFlags(&c->ev_free[b], cudaEventDisableTiming));
+    }
+    for (int i = 0; i < Ctx::kMaxEv; ++i) {
+        CK(cudaEventCreate(&c->ev[i][0]));
+        CK(cudaEventCreate(&c->ev[i][1]));
+    }
+    c->flags = env_int("ARCV_FLAGS", 0);
+    c->stages = env_int("ARCV_STAGES", 3);
+    if (c->stages != 2 && c->stages != 3 && c->stages != 4 && c->stages != 6) c->stages = 3;
+    const size_t smem = (size_t)c->stages * kStageBytes;
+    KernelFn kf = kernel_for_stages(c->stages);
+    CK(cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    int occ = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kf, kThreads, smem));
+    if (occ < 1) { set_error("kernel does not fit on an SM (smem %zu)", smem); return ARC_E_UNSUPPORTED; }
+    const int cap = env_int("ARCV_CTAS_PER_SM", 0);
+    c->ctas_per_sm = cap > 0 ? std::min(cap, occ) : occ;
+    e = cudaMalloc(&c->counters, 2 * sizeof(unsigned long long));
+    if (e != cudaSuccess) { cudaGetLastError(); set_error("cudaMalloc counters"); return ARC_E_NOMEM; }
+    CK(cudaMemsetAsync(c->counters, 0, 2 * sizeof(unsigned long long), c->stream));
+    CK(cudaStreamSynchronize(c->stream));
+    g_ctx = c;
+    if (o.nranks > 1) {
+        int st = shard_init(*c, o.nccl_unique_id);
+        if (st) {
+            arc_verify_finalize();
+            return st;
+        }
+    }
+    return ARC_OK;
+}
+
+int arc_verify_finalize(void) {
+    if (!g_ctx) return ARC_E_NOINIT;
+    Ctx *c = g_ctx;
+    cudaStreamSynchronize(c->stream);
+    shard_finalize(*c);
+    cudaFree(c->counters);
+    cudaFree(c->status);
+    cudaFree(c->acc);
+    cudaFree(c->result_dev);
+    cudaFree(c->seg_dev);
+    cudaFree(c->report_stage);
+    cudaFree(c->packet);
+    cudaFree(c->gathered);
+    if (c->result_host) cudaFreeHost(c->result_host);
+    if (c->seg_host) cudaFreeHost(c->seg_host);
+    if (c->hdr_host) cudaFreeHost(c->hdr_host);
+    for (int b = 0; b < Ctx::kNBuf; ++b) {
+        cudaFree(c->chunk_buf[b][0]);
+        cudaFree(c->chunk_buf[b][1]);
+        cudaEventDestroy(c->ev_copy[b]);
+        cudaEventDestroy(c->ev_free[b]);
+    }
+    for (int i = 0; i < Ctx::kMaxEv; ++i) {
+        cudaEventDestroy(c->ev[i][0]);
+        cudaEventDestroy(c->ev[i][1]);
+    }
+    cudaStreamDestroy(c->copy_stream);
+    if (c->own_stream) cudaStreamDestroy(c->stream);
+    delete c;
+    g_ctx = nullptr;
+    return ARC_OK;
+}
+
+int arc_verify_set_stream(void *stream) {
+    if (!g_ctx) return ARC_E_NOINIT;
+    Ctx &c = *g_ctx;
+    if (!stream) { set_error("stream is NULL"); return ARC_E_INVAL; }
+    CK(cudaStreamSynchronize(c.stream));
+    if (c.own_stream) CK(cudaStreamDestroy(c.stream));
+    c.stream = static_cast<cudaStream_t>(stream);
+    c.own_stream = false;
+    return ARC_OK;
+}
+
+int arc_verify_set_timing(int enable) {
+    if (!g_ctx) return ARC_E_NOINIT;
+    g_ctx->timing = enable != 0;
+    return ARC_OK;
+}
+
+int arc_verify_kernel_stats(uint64_t *launches, double *total_ms, int reset) {
+    if (!g_ctx) return ARC_E_NOINIT;
+    if (launches) *launches = g_ctx->timed_launches;
+    if (total_ms) *total_ms = g_ctx->timed_ms;
+    if (reset) {
+        g_ctx->timed_launches = 0;
+        g_ctx->timed_ms = 0.0;
+    }
+    return ARC_OK;
+}
+
+int arc_verify_compare(const void *out, const void *ref, uint64_t n, arc_dtype_t dtype, double abs_tol,
+                       double rel_tol, uint64_t max_report, arc_verify_result_t *result) {
+    if (!g_ctx) return ARC_E_NOINIT;
+    arc_verify_region_t r;
+    r.out = out;
+    r.ref = ref;
+    r.n = n;
+    r.dtype = dtype;
+    r.abs_tol = abs_tol;
+    r.rel_tol = rel_tol;
+    r.max_report = max_report;
+    r.name = nullptr;
+    if (g_ctx->nranks > 1) return shard_compare(*g_ctx, r, result);
+    return run_local(*g_ctx, &r, 1, result, nullptr, true, nullptr);
+}
+
+int arc_verify_batch(const arc_verify_region_t *regions, size_t n_regions, arc_verify_result_t *results) {
+    if (!g_ctx) return ARC_E_NOINIT;
+    if (n_regions == 0) return ARC_OK;
+    if (!regions || !results) { set_error("regions/results is NULL"); return ARC_E_INVAL; }
+    return run_local(*g_ctx, regions, n_regions, results, nullptr, true, nullptr);
+}
+
+}  // extern "C"

@@ -1,0 +1,76 @@
+// arcv_internal.h -- library-private context and cross-file declarations.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "arc_verify.h"
+#include "arcv_device.cuh"
+
+namespace arcv {
+
+enum PtrKind { PK_DEVICE, PK_HOST, PK_BAD };
+
+struct Ctx {
+    static constexpr int kNBuf = 2;                       // host-input chunk ring
+    static constexpr size_t kChunkBytes = 64ull << 20;    // per array per chunk
+    static constexpr int kMaxEv = 64;
+
+    int device = 0;
+    int rank = 0, nranks = 1;
+    int num_sms = 0, ctas_per_sm = 1, stages = 3, flags = 0;
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    cudaStream_t copy_stream = nullptr;
+
+    // monotonic counters: [0] tile tickets, [1] finished CTAs (never reset;
+    // the host tracks each launch's base)
+    unsigned long long *counters = nullptr;
+    unsigned long long ticket_base = 0, done_base = 0;
+    uint16_t epoch = 0;
+
+    uint64_t *status = nullptr;        size_t status_cap = 0;
+    Acc *acc = nullptr;                size_t acc_cap = 0;
+    Acc *result_dev = nullptr;         size_t result_dev_cap = 0;
+    Acc *result_host = nullptr;        size_t result_host_cap = 0;
+    Seg *seg_dev = nullptr;            size_t seg_dev_cap = 0;
+    Seg *seg_host = nullptr;           size_t seg_host_cap = 0;
+    arc_mismatch_t *report_stage = nullptr; size_t report_stage_cap = 0;
+
+    void *chunk_buf[kNBuf][2] = {{nullptr, nullptr}, {nullptr, nullptr}};
+    cudaEvent_t ev_copy[kNBuf] = {}, ev_free[kNBuf] = {};
+    uint64_t h2d_bytes = 0;
+
+    // timing (bench)
+    bool timing = false;
+    cudaEvent_t ev[kMaxEv][2] = {};
+    int n_ev = 0;
+    uint64_t launches = 0, timed_launches = 0;
+    double timed_ms = 0.0;
+
+    // sharded mode
+    void *nccl_comm = nullptr;
+    uint8_t *packet = nullptr;         size_t packet_cap = 0;     // bytes
+    uint8_t *gathered = nullptr;       size_t gathered_cap = 0;   // bytes
+    arc_shard_header_t *hdr_host = nullptr; size_t hdr_host_cap = 0;
+    arc_shard_header_t *merge_dev = nullptr;                        // [1 + nranks] global + per-rank
+};
+
+extern Ctx *g_ctx;
+
+void set_error(const char *fmt, ...);
+int cuda_fail(cudaError_t e, const char *what);
+PtrKind classify(const void *p, int device);
+int validate_region(const void *out, const void *ref, uint64_t n, int dtype, double abs_tol, double rel_tol,
+                    uint64_t max_report, const arc_verify_result_t *res);
+int launch_segments(Ctx &c, const Seg *segs, uint32_t n_segs, uint64_t total_tiles, uint32_t acc_lo,
+                    uint32_t n_acc, bool finalize);
+int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_result_t *results,
+              arc_mismatch_t *const *dev_reports, bool d2h_reports, Acc *summaries_out);
+
+// arcv_shard.cu
+int shard_init(Ctx &c, const void *nccl_unique_id);
+void shard_finalize(Ctx &c);
+int shard_compare(Ctx &c, const arc_verify_region_t &r, arc_verify_result_t *result);
+
+}  // namespace arcv

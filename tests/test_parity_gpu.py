@@ -1,0 +1,356 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Bar: bit-exact -- mismatch count, n_reported, the bit patterns of max_abs_err /
+max_rel_err, and every report entry (index, out bits, ref bits) -- on the same
+seeded inputs (synth/), for every dtype, size class, alignment, batching,
+host/device placement and shard count.
+"""
+import os
+import struct
+
+import numpy as np
+import pytest
+import torch
+
+import synth
+
+pytestmark = pytest.mark.gpu
+
+NP = {"f32": np.float32, "f64": np.float64, "i32": np.int32, "i64": np.int64, "u8": np.uint8}
+TD = synth.TORCH_DTYPES
+TILE_ELEMS = {"f32": 4096, "f64": 2048, "i32": 4096, "i64": 2048, "u8": 16384}
+
+
+def bits(x: float) -> int:
+    return struct.unpack("<Q", struct.pack("<d", x))[0]
+
+
+def assert_same(g, o, what=""):
+    assert g.n == o.n, what
+    assert g.n_mismatch == o.n_mismatch, what
+    assert g.n_reported == o.n_reported, what
+    assert bits(g.max_abs_err) == bits(o.max_abs_err), (what, g.max_abs_err, o.max_abs_err)
+    assert bits(g.max_rel_err) == bits(o.max_rel_err), (what, g.max_rel_err, o.max_rel_err)
+    rep = g.report
+    if isinstance(rep, torch.Tensor):
+        rep = rep.cpu().numpy().view(o.report.dtype)[: g.n_reported]
+    assert np.array_equal(np.asarray(rep[: g.n_reported]), o.report), what
+
+
+@pytest.fixture(scope="module")
+def av():
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    import paper_conf_ipps_leelv14_b200 as av
+
+    av.init(0)
+    yield av
+    av.finalize()
+
+
+@pytest.fixture(scope="module")
+def orc():
+    import oracle
+
+    oracle.build()
+    return oracle
+
+
+def run_both(av, orc, out, ref, dt, at, rt, mr, what=""):
+    g = av.compare(out, ref, at, rt, mr)
+    o = orc.compare(out.cpu().numpy(), ref.cpu().numpy(), dt, at, rt, mr)
+    assert_same(g, o, what)
+    return g, o
+
+
+def random_pair(dt, n, seed, rate=0.01, device="cuda"):
+    gen = torch.Generator(device="cpu").manual_seed(seed)
+    if dt in ("f32", "f64"):
+        ref = (torch.rand(n, generator=gen, dtype=torch.float64) * 4 - 2).to(TD[dt])
+        ibits = torch.int32 if dt == "f32" else torch.int64
+        k = torch.randint(-90, 90, (n,), generator=gen).to(ibits)
+        out = (ref.view(ibits) + k).view(TD[dt])
+        m = torch.rand(n, generator=gen) < rate
+        out[m] = out[m] * 1.5 + 0.25
+    else:
+        hi = 255 if dt == "u8" else 1 << 30
+        ref = torch.randint(0, hi, (n,), generator=gen).to(TD[dt])
+        out = ref.clone()
+        m = torch.rand(n, generator=gen) < rate
+        out[m] = (out[m] ^ 3) if dt != "u8" else (out[m] ^ 3)
+    return out.to(device), ref.to(device)
+
+
+# ------------------------------------------------------------------ configs
+def test_c1(av, orc):
+    c1 = synth.C1()
+    out, ref = c1.slice()
+    g, o = run_both(av, orc, out.cuda(), ref.cuda(), "f32", c1.abs_tol, c1.rel_tol, c1.max_report, "C1")
+    assert g.n_mismatch == 45 and list(g.report["index"]) == c1.planted()
+
+
+@pytest.mark.parametrize("tol", synth.TOL_PAIRS)
+def test_special_pairs(av, orc, tol):
+    sp = np.array(synth.F32_SPECIAL_BITS, dtype=np.uint32).view(np.float32)
+    out = torch.from_numpy(np.repeat(sp, sp.size)).cuda()
+    ref = torch.from_numpy(np.tile(sp, sp.size)).cuda()
+    run_both(av, orc, out, ref, "f32", tol[0], tol[1], 10 ** 6, f"specials {tol}")
+    # the same values widened to fp64 inputs
+    run_both(av, orc, out.double(), ref.double(), "f64", tol[0], tol[1], 10 ** 6, f"specials64 {tol}")
+
+
+def test_subnormal_canary(av, orc):
+    """fp32 subnormals must not be flushed by the widening (reading R8)."""
+    out = torch.tensor([1.4e-45, 1.1754942e-38, -1.4e-45], dtype=torch.float32).cuda()
+    ref = torch.zeros(3, dtype=torch.float32).cuda()
+    g, _ = run_both(av, orc, out, ref, "f32", 0.0, 0.0, 8)
+    assert g.n_mismatch == 3 and g.max_abs_err == float(np.float32(1.1754942e-38))
+
+
+@pytest.mark.parametrize("variant", ["A", "B"])
+def test_c2(av, orc, variant):
+    c2 = synth.C2(variant)
+    out, ref = c2.slice(device="cuda")
+    g, _ = run_both(av, orc, out, ref, "f32", c2.abs_tol, c2.rel_tol, c2.max_report, f"C2{variant}")
+    assert list(g.report["index"]) == c2.planted()
+
+
+# ----------------------------------------------------- sizes / alignment
+def _sizes(dt):
+    te = TILE_ELEMS[dt]
+    return sorted({0, 1, 2, 7, 31, 33, 255, te - 1, te, te + 1, 3 * te + 17, 148 * 3 * te + 5, (1 << 20) + 1})
+
+
+@pytest.mark.parametrize("dt", ["f32", "f64", "i32", "i64", "u8"])
+def test_sizes_and_misalignment(av, orc, dt):
+    for n in _sizes(dt):
+        for off in (0, 1, 3) if n < 1 << 16 else (0, 1):
+            big_o, big_r = random_pair(dt, n + off + 3, seed=n * 7 + off)
+            out, ref = big_o[off:off + n], big_r[off:off + n]  # storage offset -> misaligned windows
+            for mr in (0, 1, 64, 10 ** 9):
+                run_both(av, orc, out, ref, dt, 1e-6, 1e-5, mr, f"{dt} n={n} off={off} mr={mr}")
+
+
+@pytest.mark.parametrize("dt", ["f32", "i32", "u8"])
+def test_all_mismatch_and_report_limits(av, orc, dt):
+    n = 3 * TILE_ELEMS[dt] + 11
+    _, ref = random_pair(dt, n, seed=5, rate=0.0)
+    out = ref + 1 if dt != "u8" else (ref ^ 1)
+    for mr in (1, n - 1, n, n + 5):
+        run_both(av, orc, out, ref, dt, 0.0, 0.0, mr, f"all-mismatch {dt} mr={mr}")
+
+
+def test_aliasing(av, orc):
+    c1 = synth.C1()
+    out, _ = c1.slice()
+    out = out.cuda()
+    g, _ = run_both(av, orc, out, out, "f32", 0.0, 0.0, 100)
+    assert g.n_mismatch == 0  # NaN matches itself (rule 2)
+
+
+def test_device_report(av, orc):
+    c1 = synth.C1()
+    out, ref = c1.slice()
+    out, ref = out.cuda(), ref.cuda()
+    rep = torch.zeros(100 * 24, dtype=torch.uint8, device="cuda")
+    g = av.compare(out, ref, c1.abs_tol, c1.rel_tol, 100, report=rep)
+    o = orc.compare(out.cpu().numpy(), ref.cpu().numpy(), "f32", c1.abs_tol, c1.rel_tol, 100)
+    assert_same(g, o)
+
+
+def test_repeated_calls_are_stable(av, orc):
+    c1 = synth.C1()
+    out, ref = c1.slice()
+    out, ref = out.cuda(), ref.cuda()
+    o = orc.compare(out.cpu().numpy(), ref.cpu().numpy(), "f32", 1e-6, 1e-5, 40)
+    o2 = orc.compare(out[:5000].cpu().numpy(), ref[:5000].cpu().numpy(), "f32", 1e-6, 1e-5, 3)
+    for _ in range(40):
+        assert_same(av.compare(out, ref, 1e-6, 1e-5, 40), o)
+        assert_same(av.compare(out[:5000], ref[:5000], 1e-6, 1e-5, 3), o2)
+
+
+# ------------------------------------------------------------------ batch
+def _c3_tensors(device="cuda"):
+    regs = synth.c3_regions()
+    return regs, [(r, *r.slice(device=device)) for r in regs]
+
+
+def test_c3_batch_matches_oracle_and_singles(av, orc):
+    regs, data = _c3_tensors()
+    res = av.batch([(o, r, reg.abs_tol, reg.rel_tol, reg.max_report, reg.name) for reg, o, r in data])
+    for (reg, o, r), g in zip(data, res):
+        exp = orc.compare(o.cpu().numpy(), r.cpu().numpy(), reg.dtype, reg.abs_tol, reg.rel_tol, reg.max_report)
+        assert_same(g, exp, reg.name)
+        assert list(g.report["index"]) == reg.planted()
+        single = av.compare(o, r, reg.abs_tol, reg.rel_tol, reg.max_report)
+        assert_same(single, exp, reg.name + " single")
+
+
+def test_c3_batch_misaligned_packing(av, orc):
+    """All twelve regions packed into one byte buffer at odd element offsets."""
+    regs, data = _c3_tensors()
+    total = sum((o.numel() + 3) * o.element_size() + 64 for _, o, _ in data)
+    bo = torch.zeros(total, dtype=torch.uint8, device="cuda")
+    br = torch.zeros(total, dtype=torch.uint8, device="cuda")
+    views, pos = [], 0
+    for k, (reg, o, r) in enumerate(data):
+        es = o.element_size()
+        pos = (pos + 15) // 16 * 16 + es * (1 + 2 * (k % 3))  # odd element offset from 16B
+        nb = o.numel() * es
+        bo[pos:pos + nb].copy_(o.view(torch.uint8))
+        br[pos:pos + nb].copy_(r.view(torch.uint8))
+        views.append((reg, bo[pos:pos + nb].view(o.dtype), br[pos:pos + nb].view(o.dtype)))
+        pos += nb
+    res = av.batch([(o, r, reg.abs_tol, reg.rel_tol, 7, reg.name) for reg, o, r in views])
+    for (reg, o, r), g in zip(views, res):
+        exp = orc.compare(o.cpu().numpy(), r.cpu().numpy(), reg.dtype, reg.abs_tol, reg.rel_tol, 7)
+        assert_same(g, exp, reg.name)
+
+
+def test_batch_many_regions_table_path(av, orc):
+    """> 8 segments go through the device descriptor table; include empty regions."""
+    items, exps = [], []
+    for k in range(37):
+        dt = ["f32", "f64", "i32", "i64", "u8"][k % 5]
+        n = [0, 1, 5000, 40000, 4097][k % 5] + k
+        o, r = random_pair(dt, n, seed=100 + k, rate=0.02)
+        items.append((o, r, 1e-6, 1e-5, [0, 3, 1000][k % 3]))
+        exps.append(orc.compare(o.cpu().numpy(), r.cpu().numpy(), dt, 1e-6, 1e-5, [0, 3, 1000][k % 3]))
+    for g, e in zip(av.batch(items), exps):
+        assert_same(g, e)
+
+
+# ----------------------------------------------------------- host inputs
+@pytest.mark.parametrize("where", ["ref_pinned", "both_pinned", "ref_pageable"])
+def test_host_inputs_streamed(av, orc, where):
+    n = 40_000_003  # > 2 chunks of 64 MiB fp32
+    c = synth.C4(n)  # fp64 recipe at a smaller n
+    out, ref = c.slice(device="cuda")
+    o = orc.compare(out.cpu().numpy(), ref.cpu().numpy(), "f64", c.abs_tol, c.rel_tol, 300)
+    if where == "ref_pinned":
+        a, b = out, ref.cpu().pin_memory()
+    elif where == "both_pinned":
+        a, b = out.cpu().pin_memory(), ref.cpu().pin_memory()
+    else:
+        a, b = out, ref.cpu()
+    g = av.compare(a, b, c.abs_tol, c.rel_tol, 300)
+    assert_same(g, o, where)
+
+
+# ------------------------------------------------------------ stage variants
+@pytest.mark.parametrize("stages,ctas", [(2, 0), (4, 0), (6, 0), (3, 1)])
+def test_launch_geometry_invariance(orc, stages, ctas):
+    import paper_conf_ipps_leelv14_b200 as av
+
+    av.finalize()
+    os.environ["ARCV_STAGES"], os.environ["ARCV_CTAS_PER_SM"] = str(stages), str(ctas)
+    try:
+        av.init(0)
+        c1 = synth.C1()
+        out, ref = c1.slice()
+        run_both(av, orc, out.cuda(), ref.cuda(), "f32", 1e-6, 1e-5, 30, f"stages={stages}")
+        o5, r5 = synth.C5(1 << 22).slice(device="cuda")
+        run_both(av, orc, o5, r5, "i32", 0, 0, 5000, f"c5 stages={stages}")
+    finally:
+        av.finalize()
+        del os.environ["ARCV_STAGES"], os.environ["ARCV_CTAS_PER_SM"]
+        av.init(0)
+
+
+# --------------------------------------------------------------- full sizes
+def test_c4_full_size(av, orc):
+    c4 = synth.C4()
+    out, ref = c4.slice(device="cuda")
+    g = av.compare(out, ref, c4.abs_tol, c4.rel_tol, c4.max_report)
+    o = orc.compare(out.cpu().numpy(), ref.cpu().numpy(), "f64", c4.abs_tol, c4.rel_tol, c4.max_report)
+    assert_same(g, o, "C4")
+    assert g.n_mismatch == 516 and list(g.report["index"]) == c4.planted()
+
+
+def test_c5_full_size(av, orc):
+    c5 = synth.C5()
+    out, ref = c5.slice(device="cuda")
+    g = av.compare(out, ref, 0, 0, c5.max_report)
+    # closed form: every odd index mismatches by exactly 1
+    assert g.n_mismatch == 1 << 29 and g.n_reported == 1 << 20
+    assert g.max_abs_err == 1.0 and g.max_rel_err == 0.0
+    # the report is the oracle's on the prefix that holds the first 2^20 mismatches
+    pre = 1 << 21
+    o = orc.compare(out[:pre].cpu().numpy(), ref[:pre].cpu().numpy(), "i32", 0, 0, c5.max_report)
+    assert o.n_mismatch == 1 << 20
+    assert np.array_equal(g.report, o.report)
+
+
+def test_index_beyond_2_pow_32(av, orc):
+    n = (1 << 32) + 4099
+    ref = torch.zeros(n, dtype=torch.uint8, device="cuda")
+    out = torch.zeros(n, dtype=torch.uint8, device="cuda")
+    planted = [5, (1 << 31) + 1, (1 << 32) - 1, 1 << 32, n - 1]
+    for i in planted:
+        out[i] = 9
+    g = av.compare(out, ref, 0, 0, 100)
+    assert g.n_mismatch == len(planted) and list(g.report["index"]) == planted
+    assert g.max_abs_err == 9.0
+    tail = n - (1 << 32) + 10
+    o = orc.compare(out[-tail:].cpu().numpy(), ref[-tail:].cpu().numpy(), "u8", 0, 0, 100)
+    assert [int(i) + n - tail for i in o.report["index"]] == planted[2:]
+
+
+# ------------------------------------------------------- sharded loopback
+def _loopback(av, out, ref, dt, at, rt, mr, cuts, K):
+    p = len(cuts) - 1
+    stride = av.arc_verify_packet_bytes(K)
+    need = [av.arc_verify_packet_bytes(max(K, min(mr, b - a))) for a, b in zip(cuts[:-1], cuts[1:])]
+    gathered = torch.zeros(stride * p, dtype=torch.uint8, device="cuda")
+    code = av.DTYPE_CODES[dt]
+    for r, (a, b) in enumerate(zip(cuts[:-1], cuts[1:])):
+        pk = torch.zeros(need[r], dtype=torch.uint8, device="cuda")
+        o, f = out[a:b], ref[a:b]
+        av.arc_verify_shard_local(o.data_ptr() if b > a else 0, f.data_ptr() if b > a else 0, b - a, code,
+                                  at, rt, mr, pk.data_ptr(), K)
+        gathered[r * stride:(r + 1) * stride].copy_(pk[:stride])
+    res = av.arc_verify_result_t()
+    rep = np.zeros(max(mr, 1), dtype=av.REPORT_DTYPE)
+    res.report = rep.ctypes.data
+    av.arc_verify_shard_merge(gathered.data_ptr(), p, K, mr, res)
+    return av.Result(res.n, res.n_mismatch, res.max_abs_err, res.max_rel_err, res.n_reported, rep[: res.n_reported])
+
+
+@pytest.mark.parametrize("p", [1, 2, 3, 8])
+def test_shard_loopback_matches_unsharded(av, orc, p):
+    c1 = synth.C1()
+    out, ref = c1.slice()
+    out, ref = out.cuda(), ref.cuda()
+    n = out.numel()
+    cuts = [0] + sorted(synth.distinct_indices(7 + p, p - 1, 1, n)) + [n]
+    for mr in (0, 10, 45, 200):
+        exp = orc.compare(out.cpu().numpy(), ref.cpu().numpy(), "f32", 1e-6, 1e-5, mr)
+        g = _loopback(av, out, ref, "f32", 1e-6, 1e-5, mr, cuts, K=max(mr, 1))
+        assert_same(g, exp, f"p={p} mr={mr}")
+
+
+def test_shard_loopback_int_worst_case(av, orc):
+    c5 = synth.C5(1 << 24)
+    out, ref = c5.slice(device="cuda")
+    n = out.numel()
+    cuts = [k * n // 8 for k in range(9)]
+    mr = 1 << 20
+    exp = orc.compare(out.cpu().numpy(), ref.cpu().numpy(), "i32", 0, 0, mr)
+    g = _loopback(av, out, ref, "i32", 0, 0, mr, cuts, K=mr)
+    assert_same(g, exp, "c5 loopback")
+
+
+# ------------------------------------------------------------ bad arguments
+def test_invalid_arguments(av):
+    x = torch.zeros(16, device="cuda")
+    with pytest.raises(av.ArcVerifyError, match="invalid argument"):
+        av.compare(x, x, -1.0, 0.0, 4)
+    with pytest.raises(av.ArcVerifyError, match="invalid argument"):
+        av.compare(x, x, 0.0, float("nan"), 4)
+    xb = torch.zeros(64, dtype=torch.uint8, device="cuda")
+    mis = xb[1:33].view(torch.uint8)
+    r = av.arc_verify_result_t()
+    st = av._lib.arc_verify_compare(mis.data_ptr(), mis.data_ptr(), 8, av.ARC_F32, 0.0, 0.0, 0,
+                                    __import__("ctypes").byref(r))
+    assert st == av.ARC_E_INVAL  # fp32 pointer not 4-byte aligned
+    st = av._lib.arc_verify_compare(None, None, 8, av.ARC_F32, 0.0, 0.0, 0, __import__("ctypes").byref(r))
+    assert st == av.ARC_E_INVAL
