@@ -1,25 +1,34 @@
-// arcv_device.cuh -- sm_100a compare-reduce-compact kernel.
+// arcv_device.cuh -- sm_100a kernels of the kernel-verification comparison.
 //
-// One persistent grid streams both arrays of every segment through a
-// cp.async.bulk (TMA bulk-copy engine) ring in shared memory, evaluates the
-// element predicate of P:199 (sec. III-A; rules 1-5 in include/arc_verify.h),
-// reduces the mismatch count and the max abs/rel error, and compacts the first
-// max_report mismatches in ascending index order with a single-pass decoupled
-// look-back over per-tile mismatch counts.
+// Two kernels per verification call:
 //
-// Block = 1 producer warp (one elected lane issues the bulk copies, tile tickets
-// come from a global atomic so look-back always waits on running CTAs) + 8
-// consumer warps.  A tile is kTileBytes of EACH array; the tile's elements are
-// assigned to consumer threads in 16-byte vectors, vector v = k*256 + thread,
-// k = 0..3, so every warp's shared-memory reads are contiguous 512-byte rows.
+//  K1 arcv_stream_kernel  -- a2-a4 (+ the counting half of a5).  A persistent
+//     grid streams both arrays of every segment through a cp.async.bulk (TMA
+//     bulk-copy engine) ring in shared memory, evaluates the element predicate
+//     of P:199 (sec. III-A; rules 1-5 in include/arc_verify.h), and reduces the
+//     mismatch count and the max abs/rel error.  For regions that want a report
+//     it also records per-tile and per-group (256 tiles) mismatch counts with
+//     warp-level atomics -- no block barrier, no inter-CTA waiting in the
+//     streaming loop.
+//  K2 arcv_compact_kernel -- a5.  Scans the group and tile counts (tiny), and
+//     re-reads ONLY the tiles whose mismatches fall among the first max_report
+//     (exclusive prefix < max_report), writing their entries in ascending index
+//     order.  Sparse mismatches cost one extra tile read each; dense ones stop
+//     at max_report.  The last CTA to finish publishes the per-region summary.
 //
-// Exactness: fp32 inputs are widened exactly to fp64 (cvt.f64.f32, compiled with
-// -ftz=false so subnormals survive), the margin is __dadd_rn(abs, __dmul_rn(rel,|y|))
-// (never contracted), the division for max_rel_err is IEEE div.rn and is only
-// evaluated when it can raise the thread's running max (exact filter, DESIGN.md
-// sec. 5.3).  Maxima are order-independent, counts are integers, and the report
-// order is fixed by the element index, so the result is bit-identical to the
-// oracle for any grid, stage count, batching or chunking.
+// Block of K1 = 1 producer warp (one lane issues bulk copies; tile tickets come
+// from a global atomic so the grid is load-balanced) + 8 consumer warps.  A tile
+// is kTileBytes of EACH array; its elements are assigned to consumer threads in
+// 16-byte vectors, vector v = k*256 + thread, k = 0..3, so each warp's shared
+// memory reads are contiguous 512-byte rows.
+//
+// Exactness: float decisions are made in IEEE fp64 (cvt.f64.f32 with -ftz=false,
+// __dadd_rn(abs, __dmul_rn(rel,|y|)), never contracted, IEEE div.rn).  For fp32
+// inputs an fp32 pre-filter skips the fp64 work only when the outcome is PROVEN
+// identical (match certain, no maximum can change).  Maxima
+// are order-independent, counts are integers and the report order is fixed by
+// the element index, so results are bit-identical to the oracle for any grid,
+// stage count, batching or chunking.
 #pragma once
 #include <cstdint>
 #include <cstring>
@@ -28,78 +37,9 @@
 #include <math_constants.h>
 
 #include "arc_verify.h"
+#include "arcv_types.h"
 
 namespace arcv {
-
-constexpr int kTileBytes = 16384;                   // per array per tile
-constexpr int kSlack = 32;                          // misaligned-window slack
-constexpr int kStageArrayBytes = kTileBytes + kSlack;
-constexpr int kStageBytes = 2 * kStageArrayBytes;   // out + ref
-constexpr int kConsumerWarps = 8;
-constexpr int kConsumerThreads = kConsumerWarps * 32;
-constexpr int kThreads = kConsumerThreads + 32;     // + producer warp
-constexpr int kVecPerThread = kTileBytes / 16 / kConsumerThreads;  // 4
-constexpr int kMaxInlineSegs = 8;
-static_assert(kVecPerThread == 4, "packed-scan layout assumes 4 vectors per thread");
-
-constexpr uint64_t kValMask = (1ull << 46) - 1;     // saturating look-back value
-constexpr uint64_t kFlagA = 1ull << 46;             // tile aggregate published
-constexpr uint64_t kFlagP = 2ull << 46;             // inclusive prefix published
-constexpr int kEpochShift = 48;
-
-// One contiguous piece of one region (a whole region, or one chunk of a region
-// streamed from host memory).  96 bytes.
-struct Seg {
-    const uint8_t *out;
-    const uint8_t *ref;
-    uint64_t n;             // elements in this segment
-    uint64_t tile_begin;    // launch-local index of the segment's first tile
-    uint64_t status_begin;  // look-back status slot of the first tile
-    uint64_t chain_begin;   // status slot where this region's chain starts
-    uint64_t index_base;    // global element index of element 0
-    double abs_tol, rel_tol;
-    uint64_t max_report;    // report capacity / truncation for the region
-    arc_mismatch_t *report; // device pointer, entries [0, max_report)
-    uint32_t acc_slot;
-    uint32_t dtype;
-};
-
-struct Acc {  // per-region accumulators / result slot, 32 bytes
-    unsigned long long count;
-    unsigned long long max_abs_bits;
-    unsigned long long max_rel_bits;
-    unsigned long long pad;
-};
-
-struct Params {
-    const Seg *segs;          // device table, or nullptr -> inline_segs
-    uint32_t n_segs;
-    uint32_t n_acc;
-    uint64_t total_tiles;
-    unsigned long long *ticket;
-    unsigned long long ticket_base;
-    unsigned long long *done;
-    unsigned long long done_base;
-    uint64_t *status;
-    uint64_t epoch_tag;       // epoch << 48
-    Acc *acc;
-    Acc *result;
-    int finalize;
-    uint32_t flags;           // bit0: proxy fence before releasing a stage (diagnostic)
-    Seg inline_segs[kMaxInlineSegs];
-};
-
-struct StageInfo {
-    uint64_t tile;        // launch-local tile, ~0 = no more work
-    uint64_t elem_begin;  // segment-local index of the tile's first element
-    uint32_t seg;
-    uint32_t count;       // valid elements in the tile
-    uint32_t off_o, off_r;
-};
-
-__host__ __device__ constexpr uint32_t elem_size(uint32_t dt) {
-    return dt == ARC_F64 || dt == ARC_I64 ? 8u : (dt == ARC_U8 ? 1u : 4u);
-}
 
 // ------------------------------------------------------------------ PTX helpers
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
@@ -141,26 +81,10 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t by
 __device__ __forceinline__ void consumer_bar() {
     asm volatile("bar.sync 1, %0;" ::"n"(kConsumerThreads) : "memory");
 }
-__device__ __forceinline__ uint64_t ld_relaxed(const uint64_t *p) {
-    uint64_t v;
-    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ void st_relaxed(uint64_t *p, uint64_t v) {
-    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
 
 __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-    return v;
-}
-__device__ __forceinline__ uint64_t warp_max_u64(uint64_t v) {
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        const uint64_t w = __shfl_xor_sync(0xffffffffu, v, o);
-        v = w > v ? w : v;
-    }
     return v;
 }
 __device__ __forceinline__ double warp_max_f64(double v) {
@@ -170,21 +94,73 @@ __device__ __forceinline__ double warp_max_f64(double v) {
 }
 
 // ------------------------------------------------------------ element predicate
-// Float rules 1-5 (arc_verify.h).  Returns true on mismatch; folds d into `ma`
-// and r into `rm` (running maxima, NaN-ignoring via fmax).
-__device__ __forceinline__ bool eval_f64(double x, double y, double at, double rt, double &ma, double &rm) {
+struct ThreadAcc {
+    uint64_t count;
+    double ma, rm;     // float dtypes: running max of d and r (fp64, exact)
+    uint64_t imax;     // integer dtypes: running max |a - b|
+    float ma_rd;       // fp32 filter: RD32(ma)
+    float k_rd;        // fp32 filter: min(rt_rd, RD32(rm * (1 - 2^-40)), 0.25)
+    __device__ void reset() {
+        count = 0; ma = 0.0; rm = 0.0; imax = 0; ma_rd = 0.f; k_rd = 0.f;
+    }
+};
+
+// Float rules 1-5 (arc_verify.h), in fp64.  Returns true on mismatch; folds d
+// into acc.ma and r into acc.rm (running maxima, NaN-ignoring via fmax).
+__device__ __forceinline__ bool eval_f64(double x, double y, double at, double rt, ThreadAcc &acc) {
     const double d = fabs(x - y);             // NaN iff an operand is NaN (or Inf - Inf)
     const double ay = fabs(y);
     const double t = __dadd_rn(at, __dmul_rn(rt, ay));
     const bool match = (x == y) | ((x != x) & (y != y)) | ((ay < CUDART_INF) & (d <= t));
-    ma = fmax(ma, d);                          // rule 1: x == y -> d = 0 (or NaN for equal Inf: ignored)
+    acc.ma = fmax(acc.ma, d);                 // rule 1: x == y -> d = 0 (or NaN for equal Inf: ignored)
     // r > rm is only possible if d >= RN(rm * |y|) (monotone rounding); the
     // negated compare also lets NaN products through (rm = 0, |y| = Inf).
-    if ((d > 0.0) & !(d < rm * ay)) {
+    if ((d > 0.0) & !(d < acc.rm * ay)) {
         const double r = (ay == CUDART_INF) ? CUDART_INF : d / ay;  // rule 4 / rule 5
-        rm = fmax(rm, r);
+        acc.rm = fmax(acc.rm, r);
     }
     return !match;
+}
+
+// fp32 slow path (out of line, rare): the exact fp64 rule, then refresh the
+// filter bounds.
+__device__ __noinline__ bool eval_f32_slow(float xo, float yr, double at, double rt, float rt_rd, ThreadAcc &acc) {
+    const bool mis = eval_f64((double)xo, (double)yr, at, rt, acc);
+    acc.ma_rd = __double2float_rd(acc.ma);
+    const float rm_rd = __double2float_rd(__dmul_rd(acc.rm, 1.0 - 0x1p-40));
+    acc.k_rd = fminf(fminf(rt_rd, rm_rd), 0.25f);
+    return mis;
+}
+
+// fp32 fast path: an element is finished in fp32 iff
+//     x == y    or    (d32 < RD32(k * |y|)  and  d32 <= ma_rd),
+// with d32 = RN32(|x - y|) (one correctly rounded op on the exact difference)
+// and k = min(rt_rd, RD32(rm(1-2^-40)), 1/4).  This PROVES:
+//   match:   d32 < RD(rt_rd|y|) <= RD(at_rd + RD(rt_rd|y|)) <= t and <= RN32(t)
+//            (at_rd, rt_rd lie strictly below abs_tol, rel_tol), and RN32 is
+//            monotone, so |x - y| < t, hence d = RN64|x - y| <= t;
+//   no new max_rel: r > rm needs d >= rm|y|, hence d32 >= RD(RD32(rm(1-2^-40))|y|);
+//   no new max_abs: d32 < |y|/4 makes x - y exact (Sterbenz), so d = d32 <= ma.
+// Everything else (mismatches, NaN/Inf, zeros with abs_tol, new maxima) goes to
+// eval_f32_slow, i.e. the plain fp64 rule.
+template <int EPV>
+__device__ __forceinline__ uint32_t eval_vec_f32(const float *xo, const float *xr, double at, double rt,
+                                                 float rt_rd, ThreadAcc &acc, uint32_t valid) {
+    uint32_t slow = 0;
+#pragma unroll
+    for (int j = 0; j < EPV; ++j) {
+        const float d32 = fabsf(__fsub_rn(xo[j], xr[j]));
+        const bool fast = (xo[j] == xr[j]) | ((d32 < __fmul_rd(acc.k_rd, fabsf(xr[j]))) & (d32 <= acc.ma_rd));
+        slow |= (uint32_t)(!fast) << j;
+    }
+    slow &= valid;
+    uint32_t mis = 0;
+    if (slow) {
+#pragma unroll
+        for (int j = 0; j < EPV; ++j)
+            if ((slow >> j) & 1u) mis |= (uint32_t)eval_f32_slow(xo[j], xr[j], at, rt, rt_rd, acc) << j;
+    }
+    return mis;
 }
 
 template <typename T>
@@ -212,20 +188,14 @@ __device__ __forceinline__ uint64_t raw_bits(T v) {
     }
 }
 
-struct ThreadAcc {
-    uint64_t count;
-    double ma, rm;     // float dtypes
-    uint64_t imax;     // integer dtypes
-    __device__ void reset() { count = 0; ma = 0.0; rm = 0.0; imax = 0; }
-};
-
 // Evaluate this thread's share of one tile; returns the mismatch bit mask
 // (bit k*EPV + j <-> tile element (k*256 + ctid)*EPV + j).
 template <typename T, bool kFull, bool kAligned>
 __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *sr, uint32_t off_o, uint32_t off_r,
-                                              uint32_t cnt, int ctid, double at, double rt, ThreadAcc &acc) {
+                                              uint32_t cnt, int ctid, const Seg &g, ThreadAcc &acc) {
     constexpr int EPV = 16 / sizeof(T);
     uint64_t mask = 0;
+    const double at = g.abs_tol, rt = g.rel_tol;
 #pragma unroll
     for (int k = 0; k < kVecPerThread; ++k) {
         const uint32_t v = k * kConsumerThreads + ctid;
@@ -242,19 +212,27 @@ __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *
                 xr[j] = *reinterpret_cast<const T *>(sr + off_r + (v * EPV + j) * sizeof(T));
             }
         }
+        uint32_t valid = EPV == 32 ? 0xffffffffu : ((1u << EPV) - 1u);
+        if constexpr (!kFull) {
+            const uint32_t e0 = v * EPV;
+            valid = e0 >= cnt ? 0u : (cnt - e0 >= (uint32_t)EPV ? valid : ((1u << (cnt - e0)) - 1u));
+        }
+        if constexpr (std::is_same<T, float>::value) {
+            mask |= (uint64_t)eval_vec_f32<EPV>(xo, xr, at, rt, g.rt_rd, acc, valid) << (k * EPV);
+        } else {
 #pragma unroll
-        for (int j = 0; j < EPV; ++j) {
-            const uint32_t e = v * EPV + j;
-            if (kFull || e < cnt) {
-                bool mis;
-                if constexpr (std::is_floating_point<T>::value) {
-                    mis = eval_f64((double)xo[j], (double)xr[j], at, rt, acc.ma, acc.rm);
-                } else {
-                    const uint64_t m = int_absdiff<T>(xo[j], xr[j]);
-                    acc.imax = m > acc.imax ? m : acc.imax;
-                    mis = m != 0;
+            for (int j = 0; j < EPV; ++j) {
+                if ((valid >> j) & 1u) {
+                    bool mis;
+                    if constexpr (std::is_same<T, double>::value) {
+                        mis = eval_f64(xo[j], xr[j], at, rt, acc);
+                    } else {
+                        const uint64_t m = int_absdiff<T>(xo[j], xr[j]);
+                        acc.imax = m > acc.imax ? m : acc.imax;
+                        mis = m != 0;
+                    }
+                    mask |= (uint64_t)mis << (k * EPV + j);
                 }
-                mask |= (uint64_t)mis << (k * EPV + j);
             }
         }
     }
@@ -263,120 +241,56 @@ __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *
 
 template <typename T>
 __device__ __forceinline__ uint64_t eval_tile_dispatch(const uint8_t *so, const uint8_t *sr, const StageInfo &si,
-                                                       int ctid, double at, double rt, ThreadAcc &acc) {
+                                                       int ctid, const Seg &g, ThreadAcc &acc) {
     constexpr uint32_t TE = kTileBytes / sizeof(T);
     const bool full = si.count == TE;
     const bool aligned = (si.off_o | si.off_r) == 0;
     if (full) {
-        if (aligned) return eval_tile<T, true, true>(so, sr, 0, 0, TE, ctid, at, rt, acc);
-        return eval_tile<T, true, false>(so, sr, si.off_o, si.off_r, TE, ctid, at, rt, acc);
+        if (aligned) return eval_tile<T, true, true>(so, sr, 0, 0, TE, ctid, g, acc);
+        return eval_tile<T, true, false>(so, sr, si.off_o, si.off_r, TE, ctid, g, acc);
     }
-    if (aligned) return eval_tile<T, false, true>(so, sr, 0, 0, si.count, ctid, at, rt, acc);
-    return eval_tile<T, false, false>(so, sr, si.off_o, si.off_r, si.count, ctid, at, rt, acc);
+    if (aligned) return eval_tile<T, false, true>(so, sr, 0, 0, si.count, ctid, g, acc);
+    return eval_tile<T, false, false>(so, sr, si.off_o, si.off_r, si.count, ctid, g, acc);
 }
 
-// ------------------------------------------------------------------- look-back
-// Executed by one full warp.  Publishes the tile's aggregate, walks back over
-// predecessors (32 at a time) until an inclusive prefix is found, publishes the
-// tile's inclusive prefix and returns the exclusive prefix (all saturating at
-// `sat` = min(max_report, 2^46 - 1)).
-__device__ __forceinline__ uint64_t lookback(uint64_t *status, uint64_t slot, uint64_t chain_begin, uint64_t agg,
-                                             uint64_t sat, uint64_t tag, int lane) {
-    const uint64_t aggs = agg < sat ? agg : sat;
-    if (slot == chain_begin) {
-        if (lane == 0) st_relaxed(status + slot, tag | kFlagP | aggs);
-        return 0;
-    }
-    if (lane == 0) st_relaxed(status + slot, tag | kFlagA | aggs);
-    uint64_t excl = 0;
-    int64_t pos = (int64_t)slot - 1;
-    const uint64_t epoch = tag >> kEpochShift;
-    while (true) {
-        const int64_t idx = pos - lane;
-        const bool in_chain = idx >= (int64_t)chain_begin;
-        uint64_t val = 0;
-        uint32_t flag = 2;  // outside the chain: behaves as prefix 0
-        uint32_t spins = 0;
-        while (true) {
-            if (in_chain) {
-                const uint64_t w = ld_relaxed(status + idx);
-                flag = ((w >> kEpochShift) == epoch) ? (uint32_t)((w >> 46) & 3) : 0u;
-                val = w & kValMask;
-            }
-            const uint32_t pm = __ballot_sync(0xffffffffu, flag == 2);
-            const uint32_t xm = __ballot_sync(0xffffffffu, flag == 0);
-            const int pl = pm ? __ffs(pm) - 1 : 32;
-            const uint32_t rel = pl >= 31 ? 0xffffffffu : ((2u << pl) - 1u);
-            if (xm & rel) {
-                if (++spins > 4) __nanosleep(64);
-                continue;
-            }
-            const uint64_t v = warp_sum_u64(((rel >> lane) & 1u) ? val : 0ull);
-            excl += v;
-            excl = excl < sat ? excl : sat;
-            if (pl < 32 || excl >= sat) {
-                if (lane == 0) {
-                    const uint64_t inc = excl + aggs;
-                    st_relaxed(status + slot, tag | kFlagP | (inc < sat ? inc : sat));
-                }
-                return excl;
-            }
-            break;
-        }
-        pos -= 32;
+__device__ __forceinline__ uint64_t eval_any(const uint8_t *so, const uint8_t *sr, const StageInfo &si, int ctid,
+                                             const Seg &g, ThreadAcc &acc) {
+    switch (g.dtype) {
+        case ARC_F32: return eval_tile_dispatch<float>(so, sr, si, ctid, g, acc);
+        case ARC_F64: return eval_tile_dispatch<double>(so, sr, si, ctid, g, acc);
+        case ARC_I32: return eval_tile_dispatch<int32_t>(so, sr, si, ctid, g, acc);
+        case ARC_I64: return eval_tile_dispatch<int64_t>(so, sr, si, ctid, g, acc);
+        default: return eval_tile_dispatch<uint8_t>(so, sr, si, ctid, g, acc);
     }
 }
 
-// ------------------------------------------------------------------ compaction
-// Writes this tile's mismatches with global report rank excl + in-tile rank,
-// for ranks < max_report.  In-tile order = element index order = (k, ctid, j).
-template <typename T>
-__device__ __noinline__ void compact_tile(const Seg &g, const StageInfo &si, uint64_t mask, uint64_t excl, int ctid,
-                                          uint64_t *s_scan) {
-    constexpr int EPV = 16 / sizeof(T);
-    constexpr uint64_t kGroup = EPV == 64 ? ~0ull : ((1ull << EPV) - 1ull);
-    const int lane = ctid & 31, cw = ctid >> 5;
-    uint64_t packed = 0;
-#pragma unroll
-    for (int k = 0; k < kVecPerThread; ++k)
-        packed |= (uint64_t)__popcll(mask & (kGroup << (k * EPV))) << (16 * k);
-    uint64_t inc = packed;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const uint64_t y = __shfl_up_sync(0xffffffffu, inc, o);
-        if (lane >= o) inc += y;
-    }
-    if (lane == 31) s_scan[cw] = inc;
-    consumer_bar();
-    uint64_t wbase = 0, total = 0;
-#pragma unroll
-    for (int w = 0; w < kConsumerWarps; ++w) {
-        const uint64_t x = s_scan[w];
-        wbase += (w < cw) ? x : 0ull;
-        total += x;
-    }
-    // no trailing barrier: s_scan is rewritten only after the next tile's two
-    // look-back barriers, which every consumer thread passes after this read.
-    const uint64_t ex = wbase + inc - packed;
-    uint64_t m = mask;
-    while (m) {
-        const int b = __ffsll((long long)m) - 1;
-        m &= m - 1;
-        const int k = b / EPV, j = b % EPV;
-        uint64_t rank = ((ex >> (16 * k)) & 0xffffull) +
-                        (uint64_t)__popcll(mask & (((1ull << j) - 1ull) << (k * EPV)));
-        for (int kk = 0; kk < k; ++kk) rank += (total >> (16 * kk)) & 0xffffull;
-        const uint64_t gi = excl + rank;
-        if (gi < g.max_report) {
-            const uint64_t le = si.elem_begin + (uint64_t)((k * kConsumerThreads + ctid) * EPV + j);
-            const T *po = reinterpret_cast<const T *>(g.out) + le;
-            const T *pr = reinterpret_cast<const T *>(g.ref) + le;
-            arc_mismatch_t *dst = g.report + gi;
-            dst->index = g.index_base + le;
-            dst->out_bits = raw_bits<T>(*po);
-            dst->ref_bits = raw_bits<T>(*pr);
-        }
-    }
+// ------------------------------------------------------------ tile loading
+// Plan the bulk copies of segment-local tile `lt`: 16-byte-aligned windows that
+// cover the tile in each array (arbitrary element alignment; the extra bytes
+// lie in the same 16-byte granules as valid ones, hence in mapped pages).
+__device__ __forceinline__ void plan_tile(const Seg &g, uint64_t lt, StageInfo &si, uintptr_t &ao, uint32_t &nbo,
+                                          uintptr_t &ar, uint32_t &nbr) {
+    const uint32_t es = elem_size(g.dtype);
+    const uint64_t te = kTileBytes / es;
+    const uint64_t e0 = lt * te;
+    const uint64_t rem = g.n - e0;
+    const uint32_t cnt = (uint32_t)(rem < te ? rem : te);
+    const uintptr_t bo = reinterpret_cast<uintptr_t>(g.out) + e0 * es;
+    const uintptr_t br = reinterpret_cast<uintptr_t>(g.ref) + e0 * es;
+    ao = bo & ~(uintptr_t)15;
+    ar = br & ~(uintptr_t)15;
+    nbo = (uint32_t)(((bo + (uint64_t)cnt * es + 15) & ~(uintptr_t)15) - ao);
+    nbr = (uint32_t)(((br + (uint64_t)cnt * es + 15) & ~(uintptr_t)15) - ar);
+    si.elem_begin = e0;
+    si.count = cnt;
+    si.off_o = (uint32_t)(bo - ao);
+    si.off_r = (uint32_t)(br - ar);
+}
+
+__device__ __forceinline__ uint64_t evict_first_policy() {
+    uint64_t policy;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(policy));
+    return policy;
 }
 
 __device__ __forceinline__ uint32_t find_seg(const Seg *segs, uint32_t n, uint64_t t) {
@@ -388,25 +302,83 @@ __device__ __forceinline__ uint32_t find_seg(const Seg *segs, uint32_t n, uint64
     return lo;
 }
 
-// --------------------------------------------------------------------- kernel
+// ------------------------------------------------------------ accumulators
+// Block-wide (consumer threads) reduction of the thread accumulators into the
+// region's global accumulator slot.
+__device__ __forceinline__ void flush_acc(Acc *acc_base, uint32_t slot, uint32_t dtype, ThreadAcc &acc, int ctid,
+                                          uint64_t (*s_u)[2], double (*s_d)[2]) {
+    const int lane = ctid & 31, cw = ctid >> 5;
+    const bool is_float = dtype == ARC_F32 || dtype == ARC_F64;
+    const double mabs = is_float ? acc.ma : __ull2double_rn(acc.imax);
+    const uint64_t c = warp_sum_u64(acc.count);
+    const double wa = warp_max_f64(mabs);
+    const double wr = warp_max_f64(acc.rm);
+    if (lane == 0) {
+        s_u[cw][0] = c;
+        s_d[cw][0] = wa;
+        s_d[cw][1] = wr;
+    }
+    consumer_bar();
+    if (ctid == 0) {
+        uint64_t tc = 0;
+        double ta = 0.0, tr = 0.0;
+        for (int w = 0; w < kConsumerWarps; ++w) {
+            tc += s_u[w][0];
+            ta = fmax(ta, s_d[w][0]);
+            tr = fmax(tr, s_d[w][1]);
+        }
+        Acc *a = acc_base + slot;
+        if (tc) atomicAdd(&a->count, (unsigned long long)tc);
+        if (ta > 0.0) atomicMax(&a->max_abs_bits, (unsigned long long)__double_as_longlong(ta));
+        if (tr > 0.0) atomicMax(&a->max_rel_bits, (unsigned long long)__double_as_longlong(tr));
+    }
+    consumer_bar();
+    acc.reset();
+}
+
+// The last CTA of the launch copies the accumulators to the result slots and
+// clears them for the next call (monotonic done counter, host-tracked base).
+__device__ __forceinline__ void finalize_launch(const Params &p, int tid, int nthreads, int *s_last) {
+    if (tid == 0) {
+        __threadfence();
+        const unsigned long long prev = atomicAdd(p.done, 1ull);
+        *s_last = (prev - p.done_base) == (unsigned long long)(gridDim.x - 1);
+    }
+    if (nthreads == kConsumerThreads) consumer_bar(); else __syncthreads();
+    if (*s_last) {
+        __threadfence();
+        for (uint32_t k = tid; k < p.n_acc; k += nthreads) {
+            Acc a;
+            a.count = __ldcg(&p.acc[k].count);
+            a.max_abs_bits = __ldcg(&p.acc[k].max_abs_bits);
+            a.max_rel_bits = __ldcg(&p.acc[k].max_rel_bits);
+            a.pad = 0;
+            p.result[k] = a;
+            p.acc[k].count = 0;
+            p.acc[k].max_abs_bits = 0;
+            p.acc[k].max_rel_bits = 0;
+        }
+    }
+}
+
+// ------------------------------------------------------------------ K1: stream
 template <int S>
-__global__ void __launch_bounds__(kThreads, 2) arcv_compare_kernel(const __grid_constant__ Params p) {
+__global__ void __launch_bounds__(kThreads, 2) arcv_stream_kernel(const __grid_constant__ Params p) {
     extern __shared__ __align__(128) uint8_t smem[];
     __shared__ __align__(8) uint64_t full_bar[S];
     __shared__ __align__(8) uint64_t empty_bar[S];
     __shared__ StageInfo info[S];
-    __shared__ uint64_t s_scan[kConsumerWarps];
     __shared__ uint64_t s_red_u[kConsumerWarps][2];
     __shared__ double s_red_d[kConsumerWarps][2];
-    __shared__ uint64_t s_excl;
-    __shared__ uint32_t s_agg;
     __shared__ int s_last;
+    __shared__ uint32_t s_tile[S];
 
     const Seg *segs = p.segs ? p.segs : p.inline_segs;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) {
+            s_tile[s] = 0u;
             mbar_init(&full_bar[s], 1);
             mbar_init(&empty_bar[s], kConsumerWarps);
         }
@@ -417,8 +389,7 @@ __global__ void __launch_bounds__(kThreads, 2) arcv_compare_kernel(const __grid_
     // ------------------------------------------------------------ producer
     if (warp == 0) {
         if (lane == 0) {
-            uint64_t policy;
-            asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(policy));
+            const uint64_t policy = evict_first_policy();
             for (uint32_t i = 0;; ++i) {
                 const int s = i % S;
                 if (i >= (uint32_t)S) mbar_wait(&empty_bar[s], ((i / S) - 1) & 1);
@@ -430,23 +401,12 @@ __global__ void __launch_bounds__(kThreads, 2) arcv_compare_kernel(const __grid_
                 }
                 const uint32_t sg = find_seg(segs, p.n_segs, t);
                 const Seg &g = segs[sg];
-                const uint32_t es = elem_size(g.dtype);
-                const uint64_t te = kTileBytes / es;
-                const uint64_t e0 = (t - g.tile_begin) * te;
-                const uint64_t rem = g.n - e0;
-                const uint32_t cnt = (uint32_t)(rem < te ? rem : te);
-                const uintptr_t bo = reinterpret_cast<uintptr_t>(g.out) + e0 * es;
-                const uintptr_t br = reinterpret_cast<uintptr_t>(g.ref) + e0 * es;
-                const uintptr_t ao = bo & ~(uintptr_t)15, ar = br & ~(uintptr_t)15;
-                const uint32_t nbo = (uint32_t)(((bo + (uint64_t)cnt * es + 15) & ~(uintptr_t)15) - ao);
-                const uint32_t nbr = (uint32_t)(((br + (uint64_t)cnt * es + 15) & ~(uintptr_t)15) - ar);
                 StageInfo &si = info[s];
+                uintptr_t ao, ar;
+                uint32_t nbo, nbr;
+                plan_tile(g, t - g.tile_begin, si, ao, nbo, ar, nbr);
                 si.tile = t;
-                si.elem_begin = e0;
                 si.seg = sg;
-                si.count = cnt;
-                si.off_o = (uint32_t)(bo - ao);
-                si.off_r = (uint32_t)(br - ar);
                 uint8_t *dst = smem + (size_t)s * kStageBytes;
                 mbar_arrive_expect_tx(&full_bar[s], nbo + nbr);
                 bulk_g2s(dst, reinterpret_cast<const void *>(ao), nbo, &full_bar[s], policy);
@@ -459,39 +419,17 @@ __global__ void __launch_bounds__(kThreads, 2) arcv_compare_kernel(const __grid_
     // ------------------------------------------------------------ consumers
     const int ctid = threadIdx.x - 32;
     const int cw = warp - 1;
+    // zero the other parity's group counters and active-list length for the next
+    // launch (the previous launch that used them has completed: same stream)
+    if (blockIdx.x == 0 && ctid == 0 && p.active_cnt_zero) *p.active_cnt_zero = 0u;
+    for (uint64_t k = (uint64_t)blockIdx.x * kConsumerThreads + ctid; k < p.n_group_zero;
+         k += (uint64_t)gridDim.x * kConsumerThreads)
+        p.group_zero[k] = 0;
+
     ThreadAcc acc;
     acc.reset();
     int cur = -1;
     uint32_t cur_dtype = 0, cur_slot = 0;
-
-    auto flush = [&](uint32_t slot, uint32_t dtype) {
-        const bool is_float = dtype == ARC_F32 || dtype == ARC_F64;
-        const double mabs = is_float ? acc.ma : __ull2double_rn(acc.imax);
-        uint64_t c = warp_sum_u64(acc.count);
-        const double wa = warp_max_f64(mabs);
-        const double wr = warp_max_f64(acc.rm);
-        if (lane == 0) {
-            s_red_u[cw][0] = c;
-            s_red_d[cw][0] = wa;
-            s_red_d[cw][1] = wr;
-        }
-        consumer_bar();
-        if (ctid == 0) {
-            uint64_t tc = 0;
-            double ta = 0.0, tr = 0.0;
-            for (int w = 0; w < kConsumerWarps; ++w) {
-                tc += s_red_u[w][0];
-                ta = fmax(ta, s_red_d[w][0]);
-                tr = fmax(tr, s_red_d[w][1]);
-            }
-            Acc *a = p.acc + slot;
-            if (tc) atomicAdd(&a->count, (unsigned long long)tc);
-            if (ta > 0.0) atomicMax(&a->max_abs_bits, (unsigned long long)__double_as_longlong(ta));
-            if (tr > 0.0) atomicMax(&a->max_rel_bits, (unsigned long long)__double_as_longlong(tr));
-        }
-        consumer_bar();
-        acc.reset();
-    };
 
     for (uint32_t i = 0;; ++i) {
         const int s = i % S;
@@ -500,82 +438,259 @@ __global__ void __launch_bounds__(kThreads, 2) arcv_compare_kernel(const __grid_
         if (si.tile == ~0ull) break;
         const Seg &g = segs[si.seg];
         if ((int)si.seg != cur) {
-            if (cur >= 0 && g.acc_slot != cur_slot) flush(cur_slot, cur_dtype);
+            if (cur >= 0 && g.acc_slot != cur_slot) flush_acc(p.acc, cur_slot, cur_dtype, acc, ctid, s_red_u, s_red_d);
             cur = (int)si.seg;
             cur_dtype = g.dtype;
             cur_slot = g.acc_slot;
         }
         const uint8_t *so = smem + (size_t)s * kStageBytes;
-        const uint8_t *sr = so + kStageArrayBytes;
-        uint64_t mask;
-        switch (g.dtype) {
-            case ARC_F32: mask = eval_tile_dispatch<float>(so, sr, si, ctid, g.abs_tol, g.rel_tol, acc); break;
-            case ARC_F64: mask = eval_tile_dispatch<double>(so, sr, si, ctid, g.abs_tol, g.rel_tol, acc); break;
-            case ARC_I32: mask = eval_tile_dispatch<int32_t>(so, sr, si, ctid, 0.0, 0.0, acc); break;
-            case ARC_I64: mask = eval_tile_dispatch<int64_t>(so, sr, si, ctid, 0.0, 0.0, acc); break;
-            default: mask = eval_tile_dispatch<uint8_t>(so, sr, si, ctid, 0.0, 0.0, acc); break;
+        const uint64_t mask = eval_any(so, so + kStageArrayBytes, si, ctid, g, acc);
+        const uint32_t cnt = (uint32_t)__popcll(mask);
+        acc.count += cnt;
+        if (g.max_report != 0) {
+            // Per-tile count for K2: warps fold their counts into the stage's
+            // shared word (arrivals << 24 | count); the last warp publishes the
+            // tile (2 global atomics per tile with mismatches, none otherwise)
+            // and clears the word before the stage can be reused.
+            const uint32_t wc = __reduce_add_sync(0xffffffffu, cnt);
+            if (lane == 0) {
+                const uint32_t old = atomicAdd(&s_tile[s], (1u << 24) | wc);
+                if ((old >> 24) == kConsumerWarps - 1) {
+                    const uint32_t tc = (old & 0xffffffu) + wc;
+                    s_tile[s] = 0u;
+                    if (tc != 0) {
+                        const uint64_t lt = si.tile - g.tile_begin;
+                        atomicAdd(p.tile_cnt + g.slot_begin + lt, tc);
+                        atomicAdd(p.group_cnt + g.group_begin + lt / kGroupTiles, tc);
+                    }
+                }
+            }
         }
         if (p.flags & 1u) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty_bar[s]);  // stage may be refilled now
-        const uint32_t cnt = (uint32_t)__popcll(mask);
-        acc.count += cnt;
-
-        if (g.max_report == 0) continue;  // count-only: no ordering needed
-
-        const uint32_t wc = __reduce_add_sync(0xffffffffu, cnt);
-        if (lane == 0) s_red_u[cw][1] = wc;
-        consumer_bar();
-        if (cw == 0) {
-            uint64_t agg = lane < kConsumerWarps ? s_red_u[lane][1] : 0ull;
-            agg = warp_sum_u64(agg);
-            const uint64_t sat = g.max_report < kValMask ? g.max_report : kValMask;
-            const uint64_t slot = g.status_begin + (si.tile - g.tile_begin);
-            const uint64_t excl = lookback(p.status, slot, g.chain_begin, agg, sat, p.epoch_tag, lane);
-            if (lane == 0) {
-                s_excl = excl;
-                s_agg = (uint32_t)agg;
-            }
-        }
-        consumer_bar();
-        const uint64_t excl = s_excl;
-        const uint32_t agg = s_agg;
-        if (agg > 0 && excl < g.max_report) {
-            switch (g.dtype) {
-                case ARC_F32: compact_tile<float>(g, si, mask, excl, ctid, s_scan); break;
-                case ARC_F64: compact_tile<double>(g, si, mask, excl, ctid, s_scan); break;
-                case ARC_I32: compact_tile<int32_t>(g, si, mask, excl, ctid, s_scan); break;
-                case ARC_I64: compact_tile<int64_t>(g, si, mask, excl, ctid, s_scan); break;
-                default: compact_tile<uint8_t>(g, si, mask, excl, ctid, s_scan); break;
-            }
-        }
-        // s_excl / s_agg / s_red_u[.][1] are rewritten only after the next tile's
-        // first barrier, which every consumer passes after reading them here.
     }
-    if (cur >= 0) flush(cur_slot, cur_dtype);
+    if (cur >= 0) flush_acc(p.acc, cur_slot, cur_dtype, acc, ctid, s_red_u, s_red_d);
+    if (p.finalize) finalize_launch(p, ctid, kConsumerThreads, &s_last);
+}
 
-    if (!p.finalize) return;
-    // Last CTA to finish publishes the accumulators and clears them for the next call.
-    if (ctid == 0) {
+// --------------------------------------------------------------- K2 helpers
+// Exclusive block scan (256 threads, __syncthreads) of a u64; returns the
+// exclusive prefix, writes the block total to *total.
+__device__ __forceinline__ uint64_t block_excl_scan(uint64_t v, uint64_t *s_w, uint64_t *total) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    uint64_t inc = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint64_t y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += y;
+    }
+    if (lane == 31) s_w[w] = inc;
+    __syncthreads();
+    uint64_t base = 0, tot = 0;
+#pragma unroll
+    for (int k = 0; k < kConsumerWarps; ++k) {
+        const uint64_t x = s_w[k];
+        base += (k < w) ? x : 0ull;
+        tot += x;
+    }
+    __syncthreads();
+    *total = tot;
+    return base + inc - v;
+}
+
+// Writes this tile's mismatches with global report rank excl + in-tile rank,
+// for ranks < max_report.  In-tile order = element index order = (k, tid, j).
+template <typename T>
+__device__ __noinline__ void compact_tile(const Seg &g, const StageInfo &si, uint64_t mask, uint64_t excl,
+                                          uint64_t *s_w) {
+    constexpr int EPV = 16 / sizeof(T);
+    constexpr uint64_t kGroup = EPV == 64 ? ~0ull : ((1ull << EPV) - 1ull);
+    const int tid = threadIdx.x;
+    uint64_t packed = 0;  // 4 x 16-bit per-k counts; field totals <= 4096 (no carries)
+#pragma unroll
+    for (int k = 0; k < kVecPerThread; ++k)
+        packed |= (uint64_t)__popcll(mask & (kGroup << (k * EPV))) << (16 * k);
+    uint64_t total;
+    const uint64_t ex = block_excl_scan(packed, s_w, &total);
+    uint64_t m = mask;
+    while (m) {
+        const int b = __ffsll((long long)m) - 1;
+        m &= m - 1;
+        const int k = b / EPV, j = b % EPV;
+        uint64_t rank = ((ex >> (16 * k)) & 0xffffull) +
+                        (uint64_t)__popcll(mask & (((1ull << j) - 1ull) << (k * EPV)));
+        for (int kk = 0; kk < k; ++kk) rank += (total >> (16 * kk)) & 0xffffull;
+        const uint64_t gi = excl + rank;
+        if (gi < g.max_report) {
+            const uint64_t le = si.elem_begin + (uint64_t)((k * kConsumerThreads + tid) * EPV + j);
+            const T *po = reinterpret_cast<const T *>(g.out) + le;
+            const T *pr = reinterpret_cast<const T *>(g.ref) + le;
+            arc_mismatch_t *dst = g.report + gi;
+            dst->index = g.index_base + le;
+            dst->out_bits = raw_bits<T>(*po);
+            dst->ref_bits = raw_bits<T>(*pr);
+        }
+    }
+}
+
+// ---------------------------------------------------------------- K2: compact
+__device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+// Software grid barrier (K2 is launched cooperatively, so all CTAs are
+// co-resident).  Monotonic counter; the host tracks each launch's base.
+__device__ __forceinline__ void grid_barrier(unsigned long long *ctr, unsigned long long base) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
         __threadfence();
-        const unsigned long long prev = atomicAdd(p.done, 1ull);
-        s_last = (prev - p.done_base) == (unsigned long long)(gridDim.x - 1);
+        atomicAdd(ctr, 1ull);
+        while (ld_acquire_u64(ctr) - base < (unsigned long long)gridDim.x) __nanosleep(64);
     }
-    consumer_bar();
-    if (s_last) {
-        __threadfence();
-        for (uint32_t k = ctid; k < p.n_acc; k += kConsumerThreads) {
-            Acc a;
-            a.count = __ldcg(&p.acc[k].count);
-            a.max_abs_bits = __ldcg(&p.acc[k].max_abs_bits);
-            a.max_rel_bits = __ldcg(&p.acc[k].max_rel_bits);
-            a.pad = 0;
-            p.result[k] = a;
-            p.acc[k].count = 0;
-            p.acc[k].max_abs_bits = 0;
-            p.acc[k].max_rel_bits = 0;
+    __syncthreads();
+}
+
+__device__ __forceinline__ void compact_any(const Seg &g, const StageInfo &si, uint64_t mask, uint64_t excl,
+                                            uint64_t *s_w) {
+    switch (g.dtype) {
+        case ARC_F32: compact_tile<float>(g, si, mask, excl, s_w); break;
+        case ARC_F64: compact_tile<double>(g, si, mask, excl, s_w); break;
+        case ARC_I32: compact_tile<int32_t>(g, si, mask, excl, s_w); break;
+        case ARC_I64: compact_tile<int64_t>(g, si, mask, excl, s_w); break;
+        default: compact_tile<uint8_t>(g, si, mask, excl, s_w); break;
+    }
+}
+
+// Phase A: every CTA scans the group counters of each reporting segment (a few
+//   KB); nonzero groups are owned round-robin by their ordinal, the owner scans
+//   the group's 256 tile counts, appends every tile whose exclusive prefix is
+//   below max_report to the active list {seg, tile, prefix}, and clears the
+//   tile counts for the next call.
+// grid barrier
+// Phase B: the active tiles are spread over all CTAs; each is re-read through a
+//   2-stage bulk-copy ring, re-evaluated, and its mismatches written at report
+//   positions prefix + in-tile rank (ascending index order).
+// grid: number of SMs (cooperative launch); block: 256; dynamic smem: 2 stages.
+__global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __grid_constant__ Params p) {
+    extern __shared__ __align__(128) uint8_t smem[];
+    __shared__ __align__(8) uint64_t bar[2];
+    __shared__ uint64_t s_w[kConsumerWarps];
+    __shared__ uint32_t s_owned[kGroupTiles];
+    __shared__ uint64_t s_owned_pre[kGroupTiles];
+    __shared__ uint32_t s_n;
+    __shared__ int s_last;
+
+    const Seg *segs = p.segs ? p.segs : p.inline_segs;
+    const int tid = threadIdx.x;
+    if (tid == 0) {
+        mbar_init(&bar[0], 1);
+        mbar_init(&bar[1], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        if (blockIdx.x == 0) *p.active_cnt_zero = 0u;  // the other parity, for the next launch
+    }
+    __syncthreads();
+
+    // ------------------------------------------------------------ phase A
+    for (uint32_t sgi = 0; sgi < p.n_segs; ++sgi) {
+        const Seg &g = segs[sgi];
+        if (g.max_report == 0 || g.n == 0) continue;
+        const uint64_t ntiles = (g.n + tile_elems(g.dtype) - 1) / tile_elems(g.dtype);
+        const uint64_t ngroups = (ntiles + kGroupTiles - 1) / kGroupTiles;
+        const uint32_t *gc = p.group_cnt + g.group_begin;
+        uint64_t tot = 0;
+        for (uint64_t k = tid; k < ngroups; k += kConsumerThreads) tot += __ldcg(gc + k);
+        uint64_t total;
+        block_excl_scan(tot, s_w, &total);
+        if (total == 0) continue;  // uniform: nothing to report or to clear
+        uint64_t base = 0;
+        if (g.flags & kSegBaseFromAcc) base = __ldcg(&p.acc[g.acc_slot].count) - total;
+
+        uint64_t run = base, ord_run = 0;
+        for (uint64_t c0 = 0; c0 < ngroups; c0 += kGroupTiles) {
+            const uint64_t gi = c0 + tid;
+            const uint32_t cnt = gi < ngroups ? __ldcg(gc + gi) : 0u;
+            // pack (nonzero ordinal, count): group counts < 2^23, 256 of them < 2^31
+            const uint64_t v = ((uint64_t)(cnt != 0) << 40) | cnt;
+            uint64_t ctot;
+            const uint64_t ex = block_excl_scan(v, s_w, &ctot);
+            const uint64_t gpre = run + (ex & ((1ull << 40) - 1));
+            const uint64_t ord = ord_run + (ex >> 40);
+            if (tid == 0) s_n = 0;
+            __syncthreads();
+            if (cnt != 0 && (ord % gridDim.x) == blockIdx.x) {
+                const uint32_t k = atomicAdd(&s_n, 1u);
+                s_owned[k] = (uint32_t)gi;
+                s_owned_pre[k] = gpre;
+            }
+            __syncthreads();
+            const uint32_t n_owned = s_n;
+            run += ctot & ((1ull << 40) - 1);
+            ord_run += ctot >> 40;
+            for (uint32_t q = 0; q < n_owned; ++q) {
+                const uint64_t t0 = (uint64_t)s_owned[q] * kGroupTiles;
+                const uint64_t gp = s_owned_pre[q];
+                const uint64_t tg = ntiles - t0 < (uint64_t)kGroupTiles ? ntiles - t0 : (uint64_t)kGroupTiles;
+                uint32_t *tc = p.tile_cnt + g.slot_begin + t0;
+                const uint32_t tcnt = (uint64_t)tid < tg ? __ldcg(tc + tid) : 0u;
+                if (gp < g.max_report) {  // uniform
+                    uint64_t gtot;
+                    const uint64_t tpre = gp + block_excl_scan(tcnt, s_w, &gtot);
+                    if (tcnt != 0 && tpre < g.max_report) {
+                        const uint32_t k = atomicAdd(p.active_cnt, 1u);
+                        p.active[2 * k] = ((uint64_t)sgi << 40) | (t0 + tid);
+                        p.active[2 * k + 1] = tpre;
+                    }
+                }
+                if (tcnt != 0) tc[tid] = 0u;  // clean for the next call
+            }
+            __syncthreads();
         }
     }
+
+    grid_barrier(p.gbar, p.gbar_base);
+
+    // ------------------------------------------------------------ phase B
+    const uint32_t n_act = *(volatile uint32_t *)p.active_cnt;
+    const uint64_t policy = evict_first_policy();
+    uint32_t phase[2] = {0u, 0u};
+    auto issue = [&](uint32_t k, int st) {
+        const uint64_t a = __ldcg(p.active + 2 * k);
+        const Seg &g = segs[a >> 40];
+        StageInfo si;
+        uintptr_t ao, ar;
+        uint32_t nbo, nbr;
+        plan_tile(g, a & ((1ull << 40) - 1), si, ao, nbo, ar, nbr);
+        uint8_t *dst = smem + (size_t)st * kStageBytes;
+        mbar_arrive_expect_tx(&bar[st], nbo + nbr);
+        bulk_g2s(dst, reinterpret_cast<const void *>(ao), nbo, &bar[st], policy);
+        bulk_g2s(dst + kStageArrayBytes, reinterpret_cast<const void *>(ar), nbr, &bar[st], policy);
+    };
+    ThreadAcc dummy;
+    dummy.reset();
+    int st = 0;
+    if (blockIdx.x < n_act && tid == 0) issue(blockIdx.x, 0);
+    for (uint32_t k = blockIdx.x; k < n_act; k += gridDim.x) {
+        const uint32_t nk = k + gridDim.x;
+        if (nk < n_act && tid == 0) issue(nk, st ^ 1);  // prefetch the next active tile
+        const uint64_t a = __ldcg(p.active + 2 * k);
+        const uint64_t excl = __ldcg(p.active + 2 * k + 1);
+        const Seg &g = segs[a >> 40];
+        StageInfo si;
+        uintptr_t ao, ar;
+        uint32_t nbo, nbr;
+        plan_tile(g, a & ((1ull << 40) - 1), si, ao, nbo, ar, nbr);
+        mbar_wait(&bar[st], phase[st]);
+        phase[st] ^= 1u;
+        const uint8_t *so = smem + (size_t)st * kStageBytes;
+        const uint64_t mask = eval_any(so, so + kStageArrayBytes, si, tid, g, dummy);
+        compact_any(g, si, mask, excl, s_w);
+        __syncthreads();  // stage `st` and s_w are reused
+        st ^= 1;
+    }
+    if (p.finalize) finalize_launch(p, tid, kConsumerThreads, &s_last);
 }
 
 }  // namespace arcv

@@ -2,9 +2,9 @@
 // planning, host-input streaming, result materialisation.
 //
 // Steps of the hot path: a1 validation + dispatch happens
-// here; a2-a5 run in arcv_compare_kernel (arcv_device.cuh); a6 (summary and
-// report to the host) and a7 (one grid over many regions) are planned here; a8
-// (cross-GPU merge) lives in arcv_shard.cu.
+// here; a2-a4 run in arcv_stream_kernel and a5 in arcv_compact_kernel
+// (arcv_device.cuh); a6 (summary and report to the host) and a7 (one grid over
+// many regions) are planned here; a8 (cross-GPU merge) lives in arcv_shard.cu.
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -45,12 +45,12 @@ Ctx *g_ctx = nullptr;
 
 // ------------------------------------------------------------------ kernels
 typedef void (*KernelFn)(Params);
-static KernelFn kernel_for_stages(int s) {
+static KernelFn stream_kernel_for(int s) {
     switch (s) {
-        case 2: return arcv_compare_kernel<2>;
-        case 4: return arcv_compare_kernel<4>;
-        case 6: return arcv_compare_kernel<6>;
-        default: return arcv_compare_kernel<3>;
+        case 2: return arcv_stream_kernel<2>;
+        case 4: return arcv_stream_kernel<4>;
+        case 6: return arcv_stream_kernel<6>;
+        default: return arcv_stream_kernel<3>;
     }
 }
 
@@ -130,16 +130,75 @@ int validate_region(const void *out, const void *ref, uint64_t n, int dtype, dou
     return ARC_OK;
 }
 
+// A float strictly below v (0 when v == 0): the fp32 pre-filter's tolerance
+// bounds (arcv_device.cuh eval_f32).
+static float lower_f32(double v) {
+    if (!(v > 0.0)) return 0.f;
+    float f = (float)v;
+    if ((double)f > v) f = nextafterf(f, 0.f);
+    f = nextafterf(f, 0.f);
+    return f > 0.f ? f : 0.f;
+}
+
+static uint64_t tiles_of(uint64_t n, uint32_t dtype) {
+    const uint64_t te = tile_elems(dtype);
+    return (n + te - 1) / te;
+}
+
+static Seg make_seg(const void *out, const void *ref, uint64_t n, uint32_t dtype, double at, double rt,
+                    uint64_t max_report, arc_mismatch_t *report, uint64_t slot_begin, uint64_t index_base,
+                    uint32_t acc_slot, uint32_t flags) {
+    Seg g;
+    memset(&g, 0, sizeof(g));
+    g.out = static_cast<const uint8_t *>(out);
+    g.ref = static_cast<const uint8_t *>(ref);
+    g.n = n;
+    g.slot_begin = slot_begin;
+    g.index_base = index_base;
+    g.abs_tol = at;
+    g.rel_tol = rt;
+    g.max_report = report ? max_report : 0;
+    g.report = report;
+    g.acc_slot = acc_slot;
+    g.dtype = dtype;
+    g.flags = flags;
+    g.at_rd = lower_f32(at);
+    g.rt_rd = lower_f32(rt);
+    return g;
+}
+
 // ------------------------------------------------------------------ launch
-int launch_segments(Ctx &c, const Seg *segs, uint32_t n_segs, uint64_t total_tiles, uint32_t acc_lo,
-                    uint32_t n_acc, bool finalize) {
+// One K1 (+ K2 when any segment wants a report) over `segs`.  Fills each seg's
+// tile_begin / group_begin.  Accumulator slots [acc_lo, acc_lo + n_acc) are
+// published to the result slots when `finalize`.
+int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_t n_acc, bool finalize) {
+    uint64_t tiles = 0, groups = 0;
+    bool need_compact = false;
+    for (uint32_t k = 0; k < n_segs; ++k) {
+        segs[k].tile_begin = tiles;
+        segs[k].group_begin = groups;
+        const uint64_t t = tiles_of(segs[k].n, segs[k].dtype);
+        tiles += t;
+        if (segs[k].max_report) {
+            groups += (t + kGroupTiles - 1) / kGroupTiles;
+            need_compact = true;
+        }
+    }
+    if (tiles == 0) return ARC_OK;
+    if (groups > c.group_cap) {  // two parity halves, zeroed
+        size_t cap2 = c.group_cap * 2;
+        int st = grow_device(&c.group_cnt, &cap2, std::max<uint64_t>(groups, 1024) * 2, true, c.stream);
+        if (st) return st;
+        c.group_cap = cap2 / 2;
+    }
+    int st = ARC_OK;
     Params p;
     memset(&p, 0, sizeof(p));
     if (n_segs <= (uint32_t)kMaxInlineSegs) {
         memcpy(p.inline_segs, segs, n_segs * sizeof(Seg));
         p.segs = nullptr;
     } else {
-        int st = grow_device(&c.seg_dev, &c.seg_dev_cap, n_segs, false, c.stream);
+        st = grow_device(&c.seg_dev, &c.seg_dev_cap, n_segs, false, c.stream);
         if (st) return st;
         st = grow_pinned(&c.seg_host, &c.seg_host_cap, n_segs);
         if (st) return st;
@@ -150,33 +209,53 @@ int launch_segments(Ctx &c, const Seg *segs, uint32_t n_segs, uint64_t total_til
     }
     p.n_segs = n_segs;
     p.n_acc = n_acc;
-    p.total_tiles = total_tiles;
+    p.total_tiles = tiles;
     p.ticket = c.counters;
     p.ticket_base = c.ticket_base;
     p.done = c.counters + 1;
     p.done_base = c.done_base;
-    p.status = c.status;
-    p.epoch_tag = (uint64_t)c.epoch << kEpochShift;
+    p.tile_cnt = c.tile_cnt;
+    p.group_cnt = c.group_cnt + (size_t)c.parity * c.group_cap;
+    p.group_zero = c.group_cnt + (size_t)(c.parity ^ 1) * c.group_cap;
+    p.n_group_zero = c.group_cap;
+    p.active = c.active;
+    p.active_cnt = c.active_cnt + c.parity;
+    p.active_cnt_zero = c.active_cnt + (c.parity ^ 1);
+    p.gbar = c.counters + 2;
+    p.gbar_base = c.gbar_base;
     p.acc = c.acc + acc_lo;
     p.result = c.result_dev + acc_lo;
-    p.finalize = finalize ? 1 : 0;
+    p.finalize = (finalize && !need_compact) ? 1 : 0;
     p.flags = (uint32_t)c.flags;
 
     const uint64_t max_grid = (uint64_t)c.num_sms * (uint64_t)c.ctas_per_sm;
-    const uint32_t grid = (uint32_t)std::min<uint64_t>(total_tiles, max_grid);
+    const uint32_t grid = (uint32_t)std::min<uint64_t>(tiles, max_grid);
     const size_t smem = (size_t)c.stages * kStageBytes;
     const bool timed = c.timing && c.n_ev < Ctx::kMaxEv;
     if (timed) CK(cudaEventRecord(c.ev[c.n_ev][0], c.stream));
-    kernel_for_stages(c.stages)<<<grid, kThreads, smem, c.stream>>>(p);
+    stream_kernel_for(c.stages)<<<grid, kThreads, smem, c.stream>>>(p);
     cudaError_t e = cudaGetLastError();
-    if (e != cudaSuccess) return cuda_fail(e, "arcv_compare_kernel launch");
+    if (e != cudaSuccess) return cuda_fail(e, "arcv_stream_kernel launch");
+    c.launches++;
+    c.ticket_base += tiles + grid;
+    if (p.finalize) c.done_base += grid;
+    if (need_compact) {
+        p.finalize = finalize ? 1 : 0;
+        p.done_base = c.done_base;
+        const uint32_t grid2 = (uint32_t)c.num_sms;
+        void *args[] = {&p};
+        e = cudaLaunchCooperativeKernel((const void *)arcv_compact_kernel, dim3(grid2), dim3(kConsumerThreads), args,
+                                        2 * kStageBytes, c.stream);
+        if (e != cudaSuccess) return cuda_fail(e, "arcv_compact_kernel cooperative launch");
+        c.launches++;
+        c.gbar_base += grid2;
+        if (finalize) c.done_base += grid2;
+    }
     if (timed) {
         CK(cudaEventRecord(c.ev[c.n_ev][1], c.stream));
         c.n_ev++;
     }
-    c.launches++;
-    c.ticket_base += total_tiles + grid;
-    if (finalize) c.done_base += grid;
+    c.parity ^= 1;
     return ARC_OK;
 }
 
@@ -191,36 +270,26 @@ static int collect_timing(Ctx &c) {
     return ARC_OK;
 }
 
-static uint64_t tiles_of(uint64_t n, uint32_t dtype) {
-    const uint64_t te = kTileBytes / elem_size(dtype);
-    return (n + te - 1) / te;
-}
-
-// Prepare per-call state: epoch, workspace sizes.
-static int begin_call(Ctx &c, uint64_t status_slots, uint32_t n_acc) {
-    int st = grow_device(&c.status, &c.status_cap, std::max<uint64_t>(status_slots, 1), true, c.stream);
+// Prepare per-call workspace sizes.
+static int begin_call(Ctx &c, uint64_t tile_slots, uint32_t n_acc) {
+    int st = grow_device(&c.tile_cnt, &c.tile_cnt_cap, std::max<uint64_t>(tile_slots, 1), true, c.stream);
+    if (st) return st;
+    st = grow_device(&c.active, &c.active_cap, 2 * c.tile_cnt_cap, false, c.stream);
     if (st) return st;
     st = grow_device(&c.acc, &c.acc_cap, std::max<uint32_t>(n_acc, 1), true, c.stream);
     if (st) return st;
     st = grow_device(&c.result_dev, &c.result_dev_cap, std::max<uint32_t>(n_acc, 1), false, c.stream);
     if (st) return st;
-    st = grow_pinned(&c.result_host, &c.result_host_cap, std::max<uint32_t>(n_acc, 1));
-    if (st) return st;
-    c.epoch = (uint16_t)(c.epoch + 1);
-    if (c.epoch == 0) {  // wrapped: stale words could alias the new epoch
-        CK(cudaMemsetAsync(c.status, 0, c.status_cap * sizeof(uint64_t), c.stream));
-        c.epoch = 1;
-    }
-    return ARC_OK;
+    return grow_pinned(&c.result_host, &c.result_host_cap, std::max<uint32_t>(n_acc, 1));
 }
 
 // Stream one region whose out and/or ref live in host memory through the chunk
 // ring: H2D copies on the copy stream overlap the compare of the previous chunk.
-static int stream_region(Ctx &c, const void *out, const void *ref, bool out_dev, bool ref_dev, uint64_t n,
-                         uint32_t dtype, double at, double rt, uint64_t max_report, arc_mismatch_t *report,
-                         uint64_t status_base, uint32_t slot) {
+static int stream_region(Ctx &c, const arc_verify_region_t &r, bool out_dev, bool ref_dev,
+                         arc_mismatch_t *report, uint64_t slot_base, uint32_t acc_slot) {
+    const uint32_t dtype = (uint32_t)r.dtype;
     const uint64_t es = elem_size(dtype);
-    const uint64_t te = kTileBytes / es;
+    const uint64_t te = tile_elems(dtype);
     const uint64_t chunk_elems = std::max<uint64_t>(te, (Ctx::kChunkBytes / es) / te * te);
     if (!c.chunk_buf[0][0]) {
         for (int b = 0; b < Ctx::kNBuf; ++b)
@@ -233,14 +302,15 @@ static int stream_region(Ctx &c, const void *out, const void *ref, bool out_dev,
                 }
             }
     }
+    const uint64_t n = r.n;
     const uint64_t nchunks = (n + chunk_elems - 1) / chunk_elems;
     for (uint64_t ci = 0; ci < nchunks; ++ci) {
         const int b = (int)(ci % Ctx::kNBuf);
         const uint64_t e0 = ci * chunk_elems;
         const uint64_t ne = std::min(chunk_elems, n - e0);
         CK(cudaStreamWaitEvent(c.copy_stream, c.ev_free[b], 0));
-        const uint8_t *po = static_cast<const uint8_t *>(out) + e0 * es;
-        const uint8_t *pr = static_cast<const uint8_t *>(ref) + e0 * es;
+        const uint8_t *po = static_cast<const uint8_t *>(r.out) + e0 * es;
+        const uint8_t *pr = static_cast<const uint8_t *>(r.ref) + e0 * es;
         if (!out_dev) {
             CK(cudaMemcpyAsync(c.chunk_buf[b][0], po, ne * es, cudaMemcpyHostToDevice, c.copy_stream));
             po = static_cast<const uint8_t *>(c.chunk_buf[b][0]);
@@ -252,22 +322,9 @@ static int stream_region(Ctx &c, const void *out, const void *ref, bool out_dev,
         c.h2d_bytes += (out_dev ? 0 : ne * es) + (ref_dev ? 0 : ne * es);
         CK(cudaEventRecord(c.ev_copy[b], c.copy_stream));
         CK(cudaStreamWaitEvent(c.stream, c.ev_copy[b], 0));
-        Seg g;
-        memset(&g, 0, sizeof(g));
-        g.out = po;
-        g.ref = pr;
-        g.n = ne;
-        g.tile_begin = 0;
-        g.status_begin = status_base + e0 / te;
-        g.chain_begin = status_base;
-        g.index_base = e0;
-        g.abs_tol = at;
-        g.rel_tol = rt;
-        g.max_report = max_report;
-        g.report = report;
-        g.acc_slot = 0;
-        g.dtype = dtype;
-        int st = launch_segments(c, &g, 1, tiles_of(ne, dtype), slot, 1, ci + 1 == nchunks);
+        Seg g = make_seg(po, pr, ne, dtype, r.abs_tol, r.rel_tol, r.max_report, report, slot_base + e0 / te, e0, 0,
+                         kSegBaseFromAcc);
+        int st = launch_segments(c, &g, 1, acc_slot, 1, ci + 1 == nchunks);
         if (st) return st;
         CK(cudaEventRecord(c.ev_free[b], c.stream));
     }
@@ -285,10 +342,10 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
         arc_mismatch_t *dreport;  // device target
         bool host_report;
         uint64_t stage_off;
-        uint64_t tiles, status_base;
+        uint64_t tiles, slot_base;
     };
     std::vector<Plan> plan(R);
-    uint64_t status_slots = 0, stage_entries = 0;
+    uint64_t tile_slots = 0, stage_entries = 0;
     for (size_t k = 0; k < R; ++k) {
         const arc_verify_region_t &r = regs[k];
         int st = validate_region(r.out, r.ref, r.n, r.dtype, r.abs_tol, r.rel_tol, r.max_report, &results[k]);
@@ -305,9 +362,9 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
             pl.ref_dev = kr == PK_DEVICE;
         }
         pl.stream = !(pl.out_dev && pl.ref_dev);
-        pl.tiles = tiles_of(r.n, r.dtype);
-        pl.status_base = status_slots;
-        status_slots += pl.tiles;
+        pl.tiles = tiles_of(r.n, (uint32_t)r.dtype);
+        pl.slot_base = tile_slots;
+        tile_slots += pl.tiles;
         const uint64_t cap = std::min<uint64_t>(r.max_report, r.n);
         pl.host_report = false;
         pl.dreport = nullptr;
@@ -323,7 +380,7 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
             }
         }
     }
-    int st = begin_call(c, status_slots, (uint32_t)R);
+    int st = begin_call(c, tile_slots, (uint32_t)R);
     if (st) return st;
     if (stage_entries) {
         st = grow_device(&c.report_stage, &c.report_stage_cap, stage_entries, false, c.stream);
@@ -332,51 +389,30 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
     for (size_t k = 0; k < R; ++k)
         if (plan[k].host_report) plan[k].dreport = c.report_stage + plan[k].stage_off;
 
-    // One grid over every device-resident region (a7).
+    // accumulator slots: device-resident regions occupy [0, D) in region order,
+    // streamed regions follow (each published by its own last chunk).
+    std::vector<uint32_t> slot_of(R, 0);
     std::vector<Seg> segs;
-    std::vector<uint32_t> dev_regions;
-    uint64_t tiles = 0;
+    uint32_t next_slot = 0;
     for (size_t k = 0; k < R; ++k) {
         const arc_verify_region_t &r = regs[k];
         if (plan[k].stream || r.n == 0) continue;
-        dev_regions.push_back((uint32_t)k);
+        slot_of[k] = next_slot;
+        segs.push_back(make_seg(r.out, r.ref, r.n, (uint32_t)r.dtype, r.abs_tol, r.rel_tol, r.max_report,
+                                plan[k].dreport, plan[k].slot_base, 0, next_slot, 0));
+        next_slot++;
     }
-    // accumulator slots: device regions occupy [0, D) in region order
-    std::vector<uint32_t> slot_of(R, 0);
-    uint32_t next_slot = 0;
-    for (uint32_t k : dev_regions) slot_of[k] = next_slot++;
     const uint32_t n_dev_slots = next_slot;
     for (size_t k = 0; k < R; ++k)
         if (plan[k].stream && regs[k].n > 0) slot_of[k] = next_slot++;
-    for (uint32_t k : dev_regions) {
-        const arc_verify_region_t &r = regs[k];
-        Seg g;
-        memset(&g, 0, sizeof(g));
-        g.out = static_cast<const uint8_t *>(r.out);
-        g.ref = static_cast<const uint8_t *>(r.ref);
-        g.n = r.n;
-        g.tile_begin = tiles;
-        g.status_begin = plan[k].status_base;
-        g.chain_begin = plan[k].status_base;
-        g.index_base = 0;
-        g.abs_tol = r.abs_tol;
-        g.rel_tol = r.rel_tol;
-        g.max_report = plan[k].dreport ? r.max_report : 0;
-        g.report = plan[k].dreport;
-        g.acc_slot = slot_of[k];
-        g.dtype = (uint32_t)r.dtype;
-        segs.push_back(g);
-        tiles += plan[k].tiles;
-    }
-    if (!segs.empty()) {
-        st = launch_segments(c, segs.data(), (uint32_t)segs.size(), tiles, 0, n_dev_slots, true);
+
+    if (!segs.empty()) {  // one grid over every device-resident region (a7)
+        st = launch_segments(c, segs.data(), (uint32_t)segs.size(), 0, n_dev_slots, true);
         if (st) return st;
     }
     for (size_t k = 0; k < R; ++k) {
-        const arc_verify_region_t &r = regs[k];
-        if (!plan[k].stream || r.n == 0) continue;
-        st = stream_region(c, r.out, r.ref, plan[k].out_dev, plan[k].ref_dev, r.n, (uint32_t)r.dtype, r.abs_tol,
-                           r.rel_tol, plan[k].dreport ? r.max_report : 0, plan[k].dreport, plan[k].status_base,
+        if (!plan[k].stream || regs[k].n == 0) continue;
+        st = stream_region(c, regs[k], plan[k].out_dev, plan[k].ref_dev, plan[k].dreport, plan[k].slot_base,
                            slot_of[k]);
         if (st) return st;
     }
@@ -425,7 +461,7 @@ using namespace arcv;
 // ====================================================================== C ABI
 extern "C" {
 
-uint32_t arc_verify_version(void) { return (1u << 16) | 0u; }
+uint32_t arc_verify_version(void) { return (1u << 16) | 1u; }
 
 const char *arc_verify_strerror(int status) {
     switch (status) {
@@ -486,16 +522,19 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
     c->stages = env_int("ARCV_STAGES", 3);
     if (c->stages != 2 && c->stages != 3 && c->stages != 4 && c->stages != 6) c->stages = 3;
     const size_t smem = (size_t)c->stages * kStageBytes;
-    KernelFn kf = kernel_for_stages(c->stages);
+    KernelFn kf = stream_kernel_for(c->stages);
     CK(cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    CK(cudaFuncSetAttribute(arcv_compact_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * kStageBytes));
     int occ = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kf, kThreads, smem));
     if (occ < 1) { set_error("kernel does not fit on an SM (smem %zu)", smem); return ARC_E_UNSUPPORTED; }
     const int cap = env_int("ARCV_CTAS_PER_SM", 0);
     c->ctas_per_sm = cap > 0 ? std::min(cap, occ) : occ;
-    e = cudaMalloc(&c->counters, 2 * sizeof(unsigned long long));
+    // counters: [0] tile tickets, [1] finished CTAs, [2] K2 grid barrier, then 2 x u32 active counts
+    e = cudaMalloc(&c->counters, 4 * sizeof(unsigned long long));
     if (e != cudaSuccess) { cudaGetLastError(); set_error("cudaMalloc counters"); return ARC_E_NOMEM; }
-    CK(cudaMemsetAsync(c->counters, 0, 2 * sizeof(unsigned long long), c->stream));
+    CK(cudaMemsetAsync(c->counters, 0, 4 * sizeof(unsigned long long), c->stream));
+    c->active_cnt = reinterpret_cast<uint32_t *>(c->counters + 3);
     CK(cudaStreamSynchronize(c->stream));
     g_ctx = c;
     if (o.nranks > 1) {
@@ -514,7 +553,9 @@ int arc_verify_finalize(void) {
     cudaStreamSynchronize(c->stream);
     shard_finalize(*c);
     cudaFree(c->counters);
-    cudaFree(c->status);
+    cudaFree(c->tile_cnt);
+    cudaFree(c->active);
+    cudaFree(c->group_cnt);
     cudaFree(c->acc);
     cudaFree(c->result_dev);
     cudaFree(c->seg_dev);

@@ -5,7 +5,7 @@
 #include <cstdint>
 
 #include "arc_verify.h"
-#include "arcv_device.cuh"
+#include "arcv_types.h"
 
 namespace arcv {
 
@@ -27,9 +27,13 @@ struct Ctx {
     // the host tracks each launch's base)
     unsigned long long *counters = nullptr;
     unsigned long long ticket_base = 0, done_base = 0;
-    uint16_t epoch = 0;
 
-    uint64_t *status = nullptr;        size_t status_cap = 0;
+    uint32_t *tile_cnt = nullptr;      size_t tile_cnt_cap = 0;   // per-tile counts (kept zero)
+    uint64_t *active = nullptr;        size_t active_cap = 0;     // K2 active list (2 words / entry)
+    uint32_t *active_cnt = nullptr;                               // [2] by parity
+    unsigned long long gbar_base = 0;
+    uint32_t *group_cnt = nullptr;     size_t group_cap = 0;      // [2][group_cap], parity per K1
+    int parity = 0;
     Acc *acc = nullptr;                size_t acc_cap = 0;
     Acc *result_dev = nullptr;         size_t result_dev_cap = 0;
     Acc *result_host = nullptr;        size_t result_host_cap = 0;
@@ -63,8 +67,7 @@ int cuda_fail(cudaError_t e, const char *what);
 PtrKind classify(const void *p, int device);
 int validate_region(const void *out, const void *ref, uint64_t n, int dtype, double abs_tol, double rel_tol,
                     uint64_t max_report, const arc_verify_result_t *res);
-int launch_segments(Ctx &c, const Seg *segs, uint32_t n_segs, uint64_t total_tiles, uint32_t acc_lo,
-                    uint32_t n_acc, bool finalize);
+int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_t n_acc, bool finalize);
 int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_result_t *results,
               arc_mismatch_t *const *dev_reports, bool d2h_reports, Acc *summaries_out);
 

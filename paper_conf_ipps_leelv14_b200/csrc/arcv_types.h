@@ -1,0 +1,89 @@
+// arcv_types.h -- workspace / launch descriptors shared by host and device code.
+#pragma once
+#include <cstdint>
+
+#include "arc_verify.h"
+
+namespace arcv {
+
+constexpr int kTileBytes = 16384;                   // per array per tile
+constexpr int kSlack = 32;                          // misaligned-window slack
+constexpr int kStageArrayBytes = kTileBytes + kSlack;
+constexpr int kStageBytes = 2 * kStageArrayBytes;   // out + ref
+constexpr int kConsumerWarps = 8;
+constexpr int kConsumerThreads = kConsumerWarps * 32;
+constexpr int kThreads = kConsumerThreads + 32;     // + producer warp
+constexpr int kVecPerThread = kTileBytes / 16 / kConsumerThreads;  // 4
+constexpr int kMaxInlineSegs = 8;
+constexpr int kGroupTiles = 256;                    // tiles per group counter
+static_assert(kVecPerThread == 4, "packed-scan layout assumes 4 vectors per thread");
+static_assert(kGroupTiles == kConsumerThreads, "K2 scans one group per block pass");
+
+constexpr uint32_t kSegBaseFromAcc = 1u;  // chunk of a streamed region: prefix base = acc count - own total
+
+// One contiguous piece of one region (a whole region, or one chunk of a region
+// streamed from host memory).
+struct Seg {
+    const uint8_t *out;
+    const uint8_t *ref;
+    uint64_t n;             // elements in this segment
+    uint64_t tile_begin;    // launch-local index of the segment's first tile
+    uint64_t slot_begin;    // per-tile count slot of the first tile
+    uint64_t group_begin;   // group counter of the first tile's group
+    uint64_t index_base;    // global element index of element 0
+    double abs_tol, rel_tol;
+    uint64_t max_report;    // report capacity / truncation for the region (0 = count only)
+    arc_mismatch_t *report; // device pointer, entries [0, max_report)
+    uint32_t acc_slot;
+    uint32_t dtype;
+    uint32_t flags;
+    float at_rd, rt_rd;     // fp32 lower bounds of abs_tol / rel_tol (fp32 pre-filter)
+    uint32_t pad;
+};
+
+struct Acc {  // per-region accumulators / result slot, 32 bytes
+    unsigned long long count;
+    unsigned long long max_abs_bits;
+    unsigned long long max_rel_bits;
+    unsigned long long pad;
+};
+
+struct Params {
+    const Seg *segs;          // device table, or nullptr -> inline_segs
+    uint32_t n_segs;
+    uint32_t n_acc;
+    uint64_t total_tiles;
+    unsigned long long *ticket;
+    unsigned long long ticket_base;
+    unsigned long long *done;
+    unsigned long long done_base;
+    uint32_t *tile_cnt;       // per-tile mismatch counts (zero between calls)
+    uint32_t *group_cnt;      // per-group counts of this launch
+    uint32_t *group_zero;     // the other parity buffer, zeroed by K1 for the next launch
+    uint64_t n_group_zero;
+    uint64_t *active;         // K2 active-tile list: {seg << 40 | tile, prefix}
+    uint32_t *active_cnt;     // this launch's list length
+    uint32_t *active_cnt_zero;  // the other parity, zeroed by K2 for the next launch
+    unsigned long long *gbar; // K2 grid barrier counter (monotonic)
+    unsigned long long gbar_base;
+    Acc *acc;
+    Acc *result;
+    int finalize;
+    uint32_t flags;
+    Seg inline_segs[kMaxInlineSegs];
+};
+
+struct StageInfo {
+    uint64_t tile;        // launch-local tile, ~0 = no more work
+    uint64_t elem_begin;  // segment-local index of the tile's first element
+    uint32_t seg;
+    uint32_t count;       // valid elements in the tile
+    uint32_t off_o, off_r;
+};
+
+__host__ __device__ constexpr uint32_t elem_size(uint32_t dt) {
+    return dt == ARC_F64 || dt == ARC_I64 ? 8u : (dt == ARC_U8 ? 1u : 4u);
+}
+__host__ __device__ constexpr uint64_t tile_elems(uint32_t dt) { return kTileBytes / elem_size(dt); }
+
+}  // namespace arcv
