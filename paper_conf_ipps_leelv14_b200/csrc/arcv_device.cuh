@@ -98,10 +98,8 @@ struct ThreadAcc {
     uint64_t count;
     double ma, rm;     // float dtypes: running max of d and r (fp64, exact)
     uint64_t imax;     // integer dtypes: running max |a - b|
-    float ma_rd;       // fp32 filter: RD32(ma)
-    float k_rd;        // fp32 filter: min(rt_rd, RD32(rm * (1 - 2^-40)), 0.25)
     __device__ void reset() {
-        count = 0; ma = 0.0; rm = 0.0; imax = 0; ma_rd = 0.f; k_rd = 0.f;
+        count = 0; ma = 0.0; rm = 0.0; imax = 0;
     }
 };
 
@@ -122,45 +120,43 @@ __device__ __forceinline__ bool eval_f64(double x, double y, double at, double r
     return !match;
 }
 
-// fp32 slow path (out of line, rare): the exact fp64 rule, then refresh the
-// filter bounds.
-__device__ __noinline__ bool eval_f32_slow(float xo, float yr, double at, double rt, float rt_rd, ThreadAcc &acc) {
-    const bool mis = eval_f64((double)xo, (double)yr, at, rt, acc);
-    acc.ma_rd = __double2float_rd(acc.ma);
-    const float rm_rd = __double2float_rd(__dmul_rd(acc.rm, 1.0 - 0x1p-40));
-    acc.k_rd = fminf(fminf(rt_rd, rm_rd), 0.25f);
-    return mis;
+// Exact pre-filter.  An element is finished without the
+// fp64 rule iff
+//     x == y    or    (d_f < RD(k * |y|)  and  d_f <= ma_f)
+// where, in the element's own precision f (fp32 or fp64),
+//     d_f = RN_f(|x - y|)  (one correctly rounded op on the exact difference;
+//           for fp64 inputs this IS the oracle's d),
+//     k   = min(rel_tol_f, rm_f, 1/4)  with rel_tol_f <= rel_tol and
+//           rm_f <= rm (fp32: RD32(rel_tol) one ulp lower, RD32(rm (1 - 2^-40))),
+//     ma_f = RD_f(ma).
+// It then PROVES the fp64 rule's outcome:
+//   match   : RD(k|y|) <= RN(rel_tol|y|) <= t, and (fp32) a float <= t is
+//             <= RN32(t); RN is monotone, so |x - y| < t and d <= t;
+//   no new max_rel: RN(d/|y|) > rm needs |x - y| > rm|y| (1 - 2^-52) > k|y|
+//             >= RD(k|y|), and RN_f is monotone, so d_f >= RD(k|y|): excluded;
+//   no new max_abs: d_f < |y|/4 makes x - y exact (Sterbenz), so d = d_f <= ma.
+// Bounds only grow, so bounds read at the start of a tile are conservative.
+template <typename T>
+struct FastBounds {
+    T k, ma;
+};
+
+__device__ __forceinline__ void refresh_bounds(const ThreadAcc &acc, float rt_rd, FastBounds<float> &b) {
+    b.ma = __double2float_rd(acc.ma);
+    b.k = fminf(fminf(rt_rd, __double2float_rd(__dmul_rd(acc.rm, 1.0 - 0x1p-40))), 0.25f);
+}
+__device__ __forceinline__ void refresh_bounds(const ThreadAcc &acc, double rt, FastBounds<double> &b) {
+    b.ma = acc.ma;
+    b.k = fmin(fmin(rt, acc.rm), 0.25);
 }
 
-// fp32 fast path: an element is finished in fp32 iff
-//     x == y    or    (d32 < RD32(k * |y|)  and  d32 <= ma_rd),
-// with d32 = RN32(|x - y|) (one correctly rounded op on the exact difference)
-// and k = min(rt_rd, RD32(rm(1-2^-40)), 1/4).  This PROVES:
-//   match:   d32 < RD(rt_rd|y|) <= RD(at_rd + RD(rt_rd|y|)) <= t and <= RN32(t)
-//            (at_rd, rt_rd lie strictly below abs_tol, rel_tol), and RN32 is
-//            monotone, so |x - y| < t, hence d = RN64|x - y| <= t;
-//   no new max_rel: r > rm needs d >= rm|y|, hence d32 >= RD(RD32(rm(1-2^-40))|y|);
-//   no new max_abs: d32 < |y|/4 makes x - y exact (Sterbenz), so d = d32 <= ma.
-// Everything else (mismatches, NaN/Inf, zeros with abs_tol, new maxima) goes to
-// eval_f32_slow, i.e. the plain fp64 rule.
-template <int EPV>
-__device__ __forceinline__ uint32_t eval_vec_f32(const float *xo, const float *xr, double at, double rt,
-                                                 float rt_rd, ThreadAcc &acc, uint32_t valid) {
-    uint32_t slow = 0;
-#pragma unroll
-    for (int j = 0; j < EPV; ++j) {
-        const float d32 = fabsf(__fsub_rn(xo[j], xr[j]));
-        const bool fast = (xo[j] == xr[j]) | ((d32 < __fmul_rd(acc.k_rd, fabsf(xr[j]))) & (d32 <= acc.ma_rd));
-        slow |= (uint32_t)(!fast) << j;
-    }
-    slow &= valid;
-    uint32_t mis = 0;
-    if (slow) {
-#pragma unroll
-        for (int j = 0; j < EPV; ++j)
-            if ((slow >> j) & 1u) mis |= (uint32_t)eval_f32_slow(xo[j], xr[j], at, rt, rt_rd, acc) << j;
-    }
-    return mis;
+__device__ __forceinline__ bool fast_ok(float x, float y, const FastBounds<float> &b) {
+    const float d = fabsf(__fsub_rn(x, y));
+    return (x == y) | ((d < __fmul_rd(b.k, fabsf(y))) & (d <= b.ma));
+}
+__device__ __forceinline__ bool fast_ok(double x, double y, const FastBounds<double> &b) {
+    const double d = fabs(__dsub_rn(x, y));
+    return (x == y) | ((d < __dmul_rd(b.k, fabs(y))) & (d <= b.ma));
 }
 
 template <typename T>
@@ -189,13 +185,21 @@ __device__ __forceinline__ uint64_t raw_bits(T v) {
 }
 
 // Evaluate this thread's share of one tile; returns the mismatch bit mask
-// (bit k*EPV + j <-> tile element (k*256 + ctid)*EPV + j).
+// (bit k*EPV + j <-> tile element (k*256 + ctid)*EPV + j).  Floats: a fast pass
+// over all elements with the exact pre-filter, then the fp64 rule only for the
+// (rare) flagged elements, re-read from the still-held shared-memory stage.
 template <typename T, bool kFull, bool kAligned>
 __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *sr, uint32_t off_o, uint32_t off_r,
                                               uint32_t cnt, int ctid, const Seg &g, ThreadAcc &acc) {
     constexpr int EPV = 16 / sizeof(T);
-    uint64_t mask = 0;
-    const double at = g.abs_tol, rt = g.rel_tol;
+    constexpr bool kFloat = std::is_floating_point<T>::value;
+    uint64_t mask = 0, slow = 0;
+    using RT = typename std::conditional<std::is_same<T, float>::value, float, double>::type;
+    FastBounds<RT> fb;
+    if constexpr (kFloat) {
+        if constexpr (std::is_same<T, float>::value) refresh_bounds(acc, g.rt_rd, fb);
+        else refresh_bounds(acc, g.rel_tol, fb);
+    }
 #pragma unroll
     for (int k = 0; k < kVecPerThread; ++k) {
         const uint32_t v = k * kConsumerThreads + ctid;
@@ -212,27 +216,38 @@ __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *
                 xr[j] = *reinterpret_cast<const T *>(sr + off_r + (v * EPV + j) * sizeof(T));
             }
         }
-        uint32_t valid = EPV == 32 ? 0xffffffffu : ((1u << EPV) - 1u);
+        uint32_t valid = (1u << EPV) - 1u;
         if constexpr (!kFull) {
             const uint32_t e0 = v * EPV;
             valid = e0 >= cnt ? 0u : (cnt - e0 >= (uint32_t)EPV ? valid : ((1u << (cnt - e0)) - 1u));
         }
-        if constexpr (std::is_same<T, float>::value) {
-            mask |= (uint64_t)eval_vec_f32<EPV>(xo, xr, at, rt, g.rt_rd, acc, valid) << (k * EPV);
+        if constexpr (kFloat) {
+            uint32_t sl = 0;
+#pragma unroll
+            for (int j = 0; j < EPV; ++j) sl |= (uint32_t)(!fast_ok((RT)xo[j], (RT)xr[j], fb)) << j;
+            slow |= (uint64_t)(sl & valid) << (k * EPV);
         } else {
+            uint32_t mis = 0;
 #pragma unroll
             for (int j = 0; j < EPV; ++j) {
-                if ((valid >> j) & 1u) {
-                    bool mis;
-                    if constexpr (std::is_same<T, double>::value) {
-                        mis = eval_f64(xo[j], xr[j], at, rt, acc);
-                    } else {
-                        const uint64_t m = int_absdiff<T>(xo[j], xr[j]);
-                        acc.imax = m > acc.imax ? m : acc.imax;
-                        mis = m != 0;
-                    }
-                    mask |= (uint64_t)mis << (k * EPV + j);
-                }
+                const uint64_t m = ((valid >> j) & 1u) ? int_absdiff<T>(xo[j], xr[j]) : 0ull;
+                acc.imax = m > acc.imax ? m : acc.imax;
+                mis |= (uint32_t)(m != 0) << j;
+            }
+            mask |= (uint64_t)mis << (k * EPV);
+        }
+    }
+    if constexpr (kFloat) {
+        if (slow) {  // rare: mismatches, specials, new maxima
+            const double at = g.abs_tol, rt = g.rel_tol;
+            uint64_t m = slow;
+            while (m) {
+                const int b = __ffsll((long long)m) - 1;
+                m &= m - 1;
+                const uint32_t e = (uint32_t)(((b / EPV) * kConsumerThreads + ctid) * EPV + (b % EPV));
+                const T x = *reinterpret_cast<const T *>(so + off_o + e * sizeof(T));
+                const T y = *reinterpret_cast<const T *>(sr + off_r + e * sizeof(T));
+                mask |= (uint64_t)eval_f64((double)x, (double)y, at, rt, acc) << b;
             }
         }
     }

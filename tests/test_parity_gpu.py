@@ -354,3 +354,44 @@ def test_invalid_arguments(av):
     assert st == av.ARC_E_INVAL  # fp32 pointer not 4-byte aligned
     st = av._lib.arc_verify_compare(None, None, 8, av.ARC_F32, 0.0, 0.0, 0, __import__("ctypes").byref(r))
     assert st == av.ARC_E_INVAL
+
+
+# ------------------------------------------------ pre-filter boundary stress
+def _boundary(rng, n, dt):
+    if dt == "f32":
+        ref = rng.uniform(-4, 4, n).astype(np.float32)
+        ref[::17] = 0
+        k = rng.integers(-140, 140, n).astype(np.int64)
+        out = (ref.view(np.int32).astype(np.int64) + np.where(ref == 0, 0, k)).astype(np.int32).view(np.float32).copy()
+        out[::23] = rng.uniform(-2e-6, 2e-6, out[::23].size).astype(np.float32)
+    else:
+        ref = rng.uniform(-4, 4, n)
+        ref[::17] = 0
+        k = rng.integers(-1 << 34, 1 << 34, n)
+        out = (ref.view(np.int64) + np.where(ref == 0, 0, k)).view(np.float64).copy()
+        out[::23] = rng.uniform(-2e-6, 2e-6, out[::23].size)
+    return out, ref
+
+
+@pytest.mark.parametrize("dt", ["f32", "f64"])
+@pytest.mark.parametrize("tol", [(1e-6, 1e-5), (0.0, 1e-5), (1e-6, 0.0), (0.0, 0.0), (0.5, 0.3), (0.0, 3.0)])
+def test_prefilter_boundaries(av, orc, dt, tol):
+    rng = np.random.default_rng(11)
+    out, ref = _boundary(rng, 3_000_017, dt)
+    run_both(av, orc, torch.from_numpy(out).cuda(), torch.from_numpy(ref).cuda(), dt, tol[0], tol[1], 5000,
+             f"boundary {dt} {tol}")
+
+
+def test_prefilter_ulp_sweep(av, orc):
+    """Every fp32 out within +-160 ulps of a spread of refs, at several tolerances."""
+    refs = np.array([1.0, 0.75, -3.0, 1e-3, 12345.0, 1e-38, 3e38, 2.0 ** -126], dtype=np.float32)
+    k = np.arange(-160, 161)
+    outs, rs = [], []
+    for y in refs:
+        outs.append((np.int64(np.float32(y).view(np.int32)) + k).astype(np.int32).view(np.float32))
+        rs.append(np.full(k.size, y, dtype=np.float32))
+    out = np.tile(np.concatenate(outs), 50)
+    ref = np.tile(np.concatenate(rs), 50)
+    for at, rt in [(1e-6, 1e-5), (0.0, 1e-5), (0.0, 1.2e-7), (1e-40, 0.0)]:
+        run_both(av, orc, torch.from_numpy(out).cuda(), torch.from_numpy(ref).cuda(), "f32", at, rt, 100000,
+                 f"ulp sweep {at} {rt}")
