@@ -243,6 +243,11 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     ms_max, kern_avg_ms = float(t[0]), float(t[1])
 
+    # in-run read-only ceiling: the same bulk-copy pipeline with the predicate off
+    probe = None
+    if not args.profile:
+        probe = av.arc_verify_probe_read(out.data_ptr(), ref.data_ptr(), (hi - lo) * ES, iters=10)
+
     # parity of the timed result against the generator's closed form
     planted = c4.planted()
     parity = (res.n_mismatch == len(planted) and list(res.report["index"]) == planted)
@@ -297,7 +302,9 @@ def main():
             "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                          "frac": round(achieved / peak, 4), "traffic": ncu_traffic(),
                          "kernel": "arcv_stream_kernel+arcv_compact_kernel", "kernel_ms_avg": round(kern_avg_ms, 4),
-                         "algorithmic_bytes_per_launch": local_bytes, "peak_source": peak_src},
+                         "algorithmic_bytes_per_launch": local_bytes, "peak_source": peak_src,
+                         "read_probe_gbs": round(probe, 1) if probe else None,
+                         "frac_of_read_probe": round(achieved / probe, 4) if probe else None},
             "e2e": e2e,
         }
         if sampler:

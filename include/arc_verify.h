@@ -183,6 +183,16 @@ int arc_verify_get_unique_id(void *id);
 int arc_verify_set_timing(int enable);
 int arc_verify_kernel_stats(uint64_t *launches, double *total_ms, int reset);
 
+/*
+ * arc_verify_probe_read -- DIAGNOSTIC (benchmarks only, not part of the method):
+ * stream two device buffers of `bytes` each through the same bulk-copy pipeline
+ * as the comparison, with the predicate disabled, `iters` times, and return the
+ * achieved read bandwidth in GB/s (2 * bytes * iters / time).  It is the in-run
+ * read-only ceiling the comparison kernel is judged against.
+ * Errors: ARC_E_INVAL (NULL / host buffers, bytes == 0, iters < 1), ARC_E_NOINIT.
+ */
+int arc_verify_probe_read(const void *a, const void *b, uint64_t bytes, int iters, double *gbs);
+
 /* ABI version (major << 16 | minor). */
 uint32_t arc_verify_version(void);
 

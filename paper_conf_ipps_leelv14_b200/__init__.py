@@ -37,7 +37,7 @@ EXPORTED = [
     "arc_verify_strerror", "arc_verify_last_error", "arc_verify_set_stream",
     "arc_verify_get_unique_id", "arc_verify_set_timing", "arc_verify_kernel_stats",
     "arc_verify_version", "arc_verify_merge_plan", "arc_verify_packet_bytes",
-    "arc_verify_shard_local", "arc_verify_shard_merge",
+    "arc_verify_shard_local", "arc_verify_shard_merge", "arc_verify_probe_read",
 ]
 
 
@@ -101,6 +101,7 @@ def _load() -> ctypes.CDLL:
         "arc_verify_packet_bytes": (SZ, [U64]),
         "arc_verify_shard_local": (I, [P, P, U64, I, D, D, U64, P, U64]),
         "arc_verify_shard_merge": (I, [P, I, U64, U64, ctypes.POINTER(arc_verify_result_t)]),
+        "arc_verify_probe_read": (I, [P, P, U64, I, ctypes.POINTER(D)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -197,6 +198,13 @@ def arc_verify_shard_local(out_ptr, ref_ptr, n, dtype, abs_tol, rel_tol, max_rep
 def arc_verify_shard_merge(gathered_ptr, nranks, packet_entries, max_report, result: arc_verify_result_t):
     _check(_lib.arc_verify_shard_merge(gathered_ptr, nranks, packet_entries, max_report, ctypes.byref(result)),
            "arc_verify_shard_merge")
+
+
+def arc_verify_probe_read(a_ptr: int, b_ptr: int, nbytes: int, iters: int = 10) -> float:
+    """Diagnostic: read-only streaming GB/s of the comparison's pipeline (no predicate)."""
+    g = ctypes.c_double()
+    _check(_lib.arc_verify_probe_read(a_ptr, b_ptr, nbytes, iters, ctypes.byref(g)), "arc_verify_probe_read")
+    return float(g.value)
 
 
 # ------------------------------------------------------------- conveniences

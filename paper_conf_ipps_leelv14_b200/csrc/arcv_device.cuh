@@ -103,6 +103,20 @@ struct ThreadAcc {
     }
 };
 
+// The fields of the current segment that the per-tile path needs, cached in
+// registers (the Seg table lives in param / global space: generic loads).
+struct SegHot {
+    double abs_tol, rel_tol;
+    uint64_t max_report, tile_begin, slot_begin, group_begin;
+    float rt_rd;
+    uint32_t dtype, acc_slot;
+    __device__ __forceinline__ void load(const Seg &g) {
+        abs_tol = g.abs_tol; rel_tol = g.rel_tol; max_report = g.max_report;
+        tile_begin = g.tile_begin; slot_begin = g.slot_begin; group_begin = g.group_begin;
+        rt_rd = g.rt_rd; dtype = g.dtype; acc_slot = g.acc_slot;
+    }
+};
+
 // Float rules 1-5 (arc_verify.h), in fp64.  Returns true on mismatch; folds d
 // into acc.ma and r into acc.rm (running maxima, NaN-ignoring via fmax).
 __device__ __forceinline__ bool eval_f64(double x, double y, double at, double rt, ThreadAcc &acc) {
@@ -190,7 +204,7 @@ __device__ __forceinline__ uint64_t raw_bits(T v) {
 // (rare) flagged elements, re-read from the still-held shared-memory stage.
 template <typename T, bool kFull, bool kAligned>
 __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *sr, uint32_t off_o, uint32_t off_r,
-                                              uint32_t cnt, int ctid, const Seg &g, ThreadAcc &acc) {
+                                              uint32_t cnt, int ctid, const SegHot &g, ThreadAcc &acc) {
     constexpr int EPV = 16 / sizeof(T);
     constexpr bool kFloat = std::is_floating_point<T>::value;
     uint64_t mask = 0, slow = 0;
@@ -256,7 +270,7 @@ __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *
 
 template <typename T>
 __device__ __forceinline__ uint64_t eval_tile_dispatch(const uint8_t *so, const uint8_t *sr, const StageInfo &si,
-                                                       int ctid, const Seg &g, ThreadAcc &acc) {
+                                                       int ctid, const SegHot &g, ThreadAcc &acc) {
     constexpr uint32_t TE = kTileBytes / sizeof(T);
     const bool full = si.count == TE;
     const bool aligned = (si.off_o | si.off_r) == 0;
@@ -269,7 +283,7 @@ __device__ __forceinline__ uint64_t eval_tile_dispatch(const uint8_t *so, const 
 }
 
 __device__ __forceinline__ uint64_t eval_any(const uint8_t *so, const uint8_t *sr, const StageInfo &si, int ctid,
-                                             const Seg &g, ThreadAcc &acc) {
+                                             const SegHot &g, ThreadAcc &acc) {
     switch (g.dtype) {
         case ARC_F32: return eval_tile_dispatch<float>(so, sr, si, ctid, g, acc);
         case ARC_F64: return eval_tile_dispatch<double>(so, sr, si, ctid, g, acc);
@@ -377,8 +391,8 @@ __device__ __forceinline__ void finalize_launch(const Params &p, int tid, int nt
 }
 
 // ------------------------------------------------------------------ K1: stream
-template <int S>
-__global__ void __launch_bounds__(kThreads, 2) arcv_stream_kernel(const __grid_constant__ Params p) {
+template <int S, int MINB>
+__global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __grid_constant__ Params p) {
     extern __shared__ __align__(128) uint8_t smem[];
     __shared__ __align__(8) uint64_t full_bar[S];
     __shared__ __align__(8) uint64_t empty_bar[S];
@@ -444,22 +458,21 @@ __global__ void __launch_bounds__(kThreads, 2) arcv_stream_kernel(const __grid_c
     ThreadAcc acc;
     acc.reset();
     int cur = -1;
-    uint32_t cur_dtype = 0, cur_slot = 0;
+    SegHot g;
 
     for (uint32_t i = 0;; ++i) {
         const int s = i % S;
         mbar_wait(&full_bar[s], (i / S) & 1);
         const StageInfo si = info[s];
         if (si.tile == ~0ull) break;
-        const Seg &g = segs[si.seg];
         if ((int)si.seg != cur) {
-            if (cur >= 0 && g.acc_slot != cur_slot) flush_acc(p.acc, cur_slot, cur_dtype, acc, ctid, s_red_u, s_red_d);
+            const uint32_t slot = segs[si.seg].acc_slot;
+            if (cur >= 0 && slot != g.acc_slot) flush_acc(p.acc, g.acc_slot, g.dtype, acc, ctid, s_red_u, s_red_d);
             cur = (int)si.seg;
-            cur_dtype = g.dtype;
-            cur_slot = g.acc_slot;
+            g.load(segs[si.seg]);
         }
         const uint8_t *so = smem + (size_t)s * kStageBytes;
-        const uint64_t mask = eval_any(so, so + kStageArrayBytes, si, ctid, g, acc);
+        const uint64_t mask = (p.flags & kFlagProbe) ? 0ull : eval_any(so, so + kStageArrayBytes, si, ctid, g, acc);
         const uint32_t cnt = (uint32_t)__popcll(mask);
         acc.count += cnt;
         if (g.max_report != 0) {
@@ -485,7 +498,7 @@ __global__ void __launch_bounds__(kThreads, 2) arcv_stream_kernel(const __grid_c
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty_bar[s]);  // stage may be refilled now
     }
-    if (cur >= 0) flush_acc(p.acc, cur_slot, cur_dtype, acc, ctid, s_red_u, s_red_d);
+    if (cur >= 0) flush_acc(p.acc, g.acc_slot, g.dtype, acc, ctid, s_red_u, s_red_d);
     if (p.finalize) finalize_launch(p, ctid, kConsumerThreads, &s_last);
 }
 
@@ -700,7 +713,9 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
         mbar_wait(&bar[st], phase[st]);
         phase[st] ^= 1u;
         const uint8_t *so = smem + (size_t)st * kStageBytes;
-        const uint64_t mask = eval_any(so, so + kStageArrayBytes, si, tid, g, dummy);
+        SegHot gh;
+        gh.load(g);
+        const uint64_t mask = eval_any(so, so + kStageArrayBytes, si, tid, gh, dummy);
         compact_any(g, si, mask, excl, s_w);
         __syncthreads();  // stage `st` and s_w are reused
         st ^= 1;

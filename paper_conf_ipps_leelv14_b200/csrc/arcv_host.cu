@@ -45,12 +45,14 @@ Ctx *g_ctx = nullptr;
 
 // ------------------------------------------------------------------ kernels
 typedef void (*KernelFn)(Params);
+// Variants: (stages, min CTAs per SM).  Stage ring bytes per SM stay within
+// the 228 KB shared memory: 3x2 (default), 2x3, 4x1, 6x1.
 static KernelFn stream_kernel_for(int s) {
     switch (s) {
-        case 2: return arcv_stream_kernel<2>;
-        case 4: return arcv_stream_kernel<4>;
-        case 6: return arcv_stream_kernel<6>;
-        default: return arcv_stream_kernel<3>;
+        case 2: return arcv_stream_kernel<2, 3>;
+        case 4: return arcv_stream_kernel<4, 1>;
+        case 6: return arcv_stream_kernel<6, 1>;
+        default: return arcv_stream_kernel<3, 2>;
     }
 }
 
@@ -624,6 +626,40 @@ int arc_verify_compare(const void *out, const void *ref, uint64_t n, arc_dtype_t
     r.name = nullptr;
     if (g_ctx->nranks > 1) return shard_compare(*g_ctx, r, result);
     return run_local(*g_ctx, &r, 1, result, nullptr, true, nullptr);
+}
+
+int arc_verify_probe_read(const void *a, const void *b, uint64_t bytes, int iters, double *gbs) {
+    if (!g_ctx) return ARC_E_NOINIT;
+    Ctx &c = *g_ctx;
+    if (!a || !b || !gbs || iters < 1 || bytes == 0 || classify(a, c.device) != PK_DEVICE ||
+        classify(b, c.device) != PK_DEVICE) {
+        set_error("probe: device buffers, bytes > 0, iters >= 1 required");
+        return ARC_E_INVAL;
+    }
+    int st = begin_call(c, tiles_of(bytes, ARC_U8), 1);
+    if (st) return st;
+    const int saved = c.flags;
+    const bool saved_t = c.timing;
+    c.flags |= (int)kFlagProbe;
+    c.timing = false;
+    cudaEvent_t e0, e1;
+    CK(cudaEventCreate(&e0));
+    CK(cudaEventCreate(&e1));
+    Seg g = make_seg(a, b, bytes, ARC_U8, 0.0, 0.0, 0, nullptr, 0, 0, 0, 0);
+    st = launch_segments(c, &g, 1, 0, 1, true);  // warm-up
+    CK(cudaEventRecord(e0, c.stream));
+    for (int i = 0; i < iters && !st; ++i) st = launch_segments(c, &g, 1, 0, 1, true);
+    CK(cudaEventRecord(e1, c.stream));
+    CK(cudaEventSynchronize(e1));
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, e0, e1));
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    c.flags = saved;
+    c.timing = saved_t;
+    if (st) return st;
+    *gbs = 2.0 * (double)bytes * iters / (ms * 1e-3) / 1e9;
+    return ARC_OK;
 }
 
 int arc_verify_batch(const arc_verify_region_t *regions, size_t n_regions, arc_verify_result_t *results) {

@@ -19,6 +19,7 @@ constexpr int kGroupTiles = 256;                    // tiles per group counter
 static_assert(kVecPerThread == 4, "packed-scan layout assumes 4 vectors per thread");
 static_assert(kGroupTiles == kConsumerThreads, "K2 scans one group per block pass");
 
+constexpr uint32_t kFlagProbe = 2u;       // Params.flags: stream only, no predicate (read probe)
 constexpr uint32_t kSegBaseFromAcc = 1u;  // chunk of a streamed region: prefix base = acc count - own total
 
 // One contiguous piece of one region (a whole region, or one chunk of a region
