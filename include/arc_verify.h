@@ -98,7 +98,9 @@ typedef struct {
                                    non-blocking stream (the caller orders its own work);
                                    (void*)1 = cudaStreamLegacy, the legacy default stream */
     int rank, nranks;           /* sharded mode when nranks > 1                           */
-    const void *nccl_unique_id; /* 128-byte ncclUniqueId (same on all ranks) if nranks > 1 */
+    const void *nccl_unique_id; /* 128-byte ncclUniqueId (same on all ranks); required if
+                                   nranks > 1; with nranks == 1 it selects the collective
+                                   path over a 1-rank communicator                        */
 } arc_verify_opts_t;
 
 typedef struct {

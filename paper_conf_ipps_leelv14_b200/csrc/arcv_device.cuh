@@ -208,6 +208,7 @@ __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *
     constexpr int EPV = 16 / sizeof(T);
     constexpr bool kFloat = std::is_floating_point<T>::value;
     uint64_t mask = 0, slow = 0;
+    uint32_t bmax = 0;  // u8 only: byte-wise running max |a - b|
     using RT = typename std::conditional<std::is_same<T, float>::value, float, double>::type;
     FastBounds<RT> fb;
     if constexpr (kFloat) {
@@ -235,7 +236,25 @@ __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *
             const uint32_t e0 = v * EPV;
             valid = e0 >= cnt ? 0u : (cnt - e0 >= (uint32_t)EPV ? valid : ((1u << (cnt - e0)) - 1u));
         }
-        if constexpr (kFloat) {
+        if constexpr (std::is_same<T, uint8_t>::value) {
+            // bytes: SIMD-within-a-register. |a-b| per byte (vabsdiffu4), running
+            // byte-wise max (vmaxu4), and 4 mismatch bits per word from vcmpne4.
+            uint32_t wa[4], wb[4], m16 = 0;
+            memcpy(wa, xo, 16);
+            memcpy(wb, xr, 16);
+#pragma unroll
+            for (int w = 0; w < 4; ++w) {
+                if constexpr (!kFull) {  // invalid bytes compare equal: spread 4 valid bits to bytes
+                    const uint32_t vb = (valid >> (4 * w)) & 0xfu;
+                    const uint32_t bm = ((vb * 0x00204081u) & 0x01010101u) * 0xffu;
+                    wb[w] = (wb[w] & bm) | (wa[w] & ~bm);
+                }
+                const uint32_t ne = __vcmpne4(wa[w], wb[w]) & 0x01010101u;
+                m16 |= ((ne * 0x10204080u) >> 28) << (4 * w);  // byte i -> bit i
+                bmax = __vmaxu4(bmax, __vabsdiffu4(wa[w], wb[w]));
+            }
+            mask |= (uint64_t)(m16 & valid) << (k * EPV);
+        } else if constexpr (kFloat) {
             uint32_t sl = 0;
 #pragma unroll
             for (int j = 0; j < EPV; ++j) sl |= (uint32_t)(!fast_ok((RT)xo[j], (RT)xr[j], fb)) << j;
@@ -251,6 +270,11 @@ __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *
             mask |= (uint64_t)mis << (k * EPV);
         }
     }
+    if constexpr (std::is_same<T, uint8_t>::value) {
+        const uint32_t m2 = __vmaxu4(bmax, bmax >> 16);
+        const uint64_t mb = (uint64_t)max(m2 & 0xffu, (m2 >> 8) & 0xffu);
+        acc.imax = mb > acc.imax ? mb : acc.imax;
+    }
     if constexpr (kFloat) {
         if (slow) {  // rare: mismatches, specials, new maxima
             const double at = g.abs_tol, rt = g.rel_tol;
@@ -261,7 +285,12 @@ __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *
                 const uint32_t e = (uint32_t)(((b / EPV) * kConsumerThreads + ctid) * EPV + (b % EPV));
                 const T x = *reinterpret_cast<const T *>(so + off_o + e * sizeof(T));
                 const T y = *reinterpret_cast<const T *>(sr + off_r + e * sizeof(T));
+                // the bounds grew since the fast pass: a re-check clears most of a
+                // warm-up tile's flags without the fp64 rule
+                if (fast_ok((RT)x, (RT)y, fb)) continue;
                 mask |= (uint64_t)eval_f64((double)x, (double)y, at, rt, acc) << b;
+                if constexpr (std::is_same<T, float>::value) refresh_bounds(acc, g.rt_rd, fb);
+                else refresh_bounds(acc, g.rel_tol, fb);
             }
         }
     }
@@ -447,10 +476,12 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
 
     // ------------------------------------------------------------ consumers
     const int ctid = threadIdx.x - 32;
-    const int cw = warp - 1;
     // zero the other parity's group counters and active-list length for the next
     // launch (the previous launch that used them has completed: same stream)
-    if (blockIdx.x == 0 && ctid == 0 && p.active_cnt_zero) *p.active_cnt_zero = 0u;
+    if (blockIdx.x == 0 && ctid == 0 && p.active_cnt_zero) {
+        *p.active_cnt_zero = 0u;
+        *p.nz_cnt_zero = 0u;
+    }
     for (uint64_t k = (uint64_t)blockIdx.x * kConsumerThreads + ctid; k < p.n_group_zero;
          k += (uint64_t)gridDim.x * kConsumerThreads)
         p.group_zero[k] = 0;
@@ -490,6 +521,15 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
                         const uint64_t lt = si.tile - g.tile_begin;
                         atomicAdd(p.tile_cnt + g.slot_begin + lt, tc);
                         atomicAdd(p.group_cnt + g.group_begin + lt / kGroupTiles, tc);
+                        // short list of nonzero tiles for K2's pool path (checked
+                        // before the atomic so a dense call stops touching it)
+                        if (*(volatile uint32_t *)p.nz_cnt < (uint32_t)kPoolCap) {
+                            const uint32_t k = atomicAdd(p.nz_cnt, 1u);
+                            if (k < (uint32_t)kPoolCap) {
+                                p.nz_list[2 * k] = ((uint64_t)si.seg << 40) | lt;
+                                p.nz_list[2 * k + 1] = tc;
+                            }
+                        }
                     }
                 }
             }
@@ -592,24 +632,34 @@ __device__ __forceinline__ void compact_any(const Seg &g, const StageInfo &si, u
     }
 }
 
-// Phase A: every CTA scans the group counters of each reporting segment (a few
+// Two ways to find the tiles whose mismatches enter the report:
+// Pool path (the common, sparse case: K1 listed <= kPoolCap nonzero tiles):
+//   every CTA loads the short list into shared memory; entry k (round-robin)
+//   gets its exclusive prefix = sum of counts of listed tiles of the same
+//   segment with a smaller index; no group walk, no grid barrier.
+// Group path (dense: the list overflowed):
+//   Phase A: every CTA scans the group counters of each reporting segment (a few
 //   KB); nonzero groups are owned round-robin by their ordinal, the owner scans
 //   the group's 256 tile counts, appends every tile whose exclusive prefix is
-//   below max_report to the active list {seg, tile, prefix}, and clears the
-//   tile counts for the next call.
-// grid barrier
-// Phase B: the active tiles are spread over all CTAs; each is re-read through a
-//   2-stage bulk-copy ring, re-evaluated, and its mismatches written at report
-//   positions prefix + in-tile rank (ascending index order).
-// grid: number of SMs (cooperative launch); block: 256; dynamic smem: 2 stages.
+//   below max_report to the active list {seg, tile, prefix}.  Grid barrier.
+// Then each CTA re-reads its active tiles through a 2-stage bulk-copy ring,
+// re-evaluates them, and writes their mismatches at report positions
+// prefix + in-tile rank (ascending index order).  Tile counts are cleared for
+// the next call by whoever handled the tile / group.
+// grid: number of SMs (cooperative launch); block: 256;
+// dynamic smem: 2 stages + pool list (kPoolCap x 12 B).
 __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __grid_constant__ Params p) {
     extern __shared__ __align__(128) uint8_t smem[];
     __shared__ __align__(8) uint64_t bar[2];
     __shared__ uint64_t s_w[kConsumerWarps];
     __shared__ uint32_t s_owned[kGroupTiles];
     __shared__ uint64_t s_owned_pre[kGroupTiles];
+    __shared__ uint64_t s_loc_key[kPoolLocal];
+    __shared__ uint64_t s_loc_pre[kPoolLocal];
     __shared__ uint32_t s_n;
     __shared__ int s_last;
+    uint64_t *s_pkey = reinterpret_cast<uint64_t *>(smem + 2 * kStageBytes);
+    uint32_t *s_pcnt = reinterpret_cast<uint32_t *>(s_pkey + kPoolCap);
 
     const Seg *segs = p.segs ? p.segs : p.inline_segs;
     const int tid = threadIdx.x;
@@ -617,108 +667,153 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
         mbar_init(&bar[0], 1);
         mbar_init(&bar[1], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-        if (blockIdx.x == 0) *p.active_cnt_zero = 0u;  // the other parity, for the next launch
     }
     __syncthreads();
-
-    // ------------------------------------------------------------ phase A
-    for (uint32_t sgi = 0; sgi < p.n_segs; ++sgi) {
-        const Seg &g = segs[sgi];
-        if (g.max_report == 0 || g.n == 0) continue;
-        const uint64_t ntiles = (g.n + tile_elems(g.dtype) - 1) / tile_elems(g.dtype);
-        const uint64_t ngroups = (ntiles + kGroupTiles - 1) / kGroupTiles;
-        const uint32_t *gc = p.group_cnt + g.group_begin;
-        uint64_t tot = 0;
-        for (uint64_t k = tid; k < ngroups; k += kConsumerThreads) tot += __ldcg(gc + k);
-        uint64_t total;
-        block_excl_scan(tot, s_w, &total);
-        if (total == 0) continue;  // uniform: nothing to report or to clear
-        uint64_t base = 0;
-        if (g.flags & kSegBaseFromAcc) base = __ldcg(&p.acc[g.acc_slot].count) - total;
-
-        uint64_t run = base, ord_run = 0;
-        for (uint64_t c0 = 0; c0 < ngroups; c0 += kGroupTiles) {
-            const uint64_t gi = c0 + tid;
-            const uint32_t cnt = gi < ngroups ? __ldcg(gc + gi) : 0u;
-            // pack (nonzero ordinal, count): group counts < 2^23, 256 of them < 2^31
-            const uint64_t v = ((uint64_t)(cnt != 0) << 40) | cnt;
-            uint64_t ctot;
-            const uint64_t ex = block_excl_scan(v, s_w, &ctot);
-            const uint64_t gpre = run + (ex & ((1ull << 40) - 1));
-            const uint64_t ord = ord_run + (ex >> 40);
-            if (tid == 0) s_n = 0;
-            __syncthreads();
-            if (cnt != 0 && (ord % gridDim.x) == blockIdx.x) {
-                const uint32_t k = atomicAdd(&s_n, 1u);
-                s_owned[k] = (uint32_t)gi;
-                s_owned_pre[k] = gpre;
-            }
-            __syncthreads();
-            const uint32_t n_owned = s_n;
-            run += ctot & ((1ull << 40) - 1);
-            ord_run += ctot >> 40;
-            for (uint32_t q = 0; q < n_owned; ++q) {
-                const uint64_t t0 = (uint64_t)s_owned[q] * kGroupTiles;
-                const uint64_t gp = s_owned_pre[q];
-                const uint64_t tg = ntiles - t0 < (uint64_t)kGroupTiles ? ntiles - t0 : (uint64_t)kGroupTiles;
-                uint32_t *tc = p.tile_cnt + g.slot_begin + t0;
-                const uint32_t tcnt = (uint64_t)tid < tg ? __ldcg(tc + tid) : 0u;
-                if (gp < g.max_report) {  // uniform
-                    uint64_t gtot;
-                    const uint64_t tpre = gp + block_excl_scan(tcnt, s_w, &gtot);
-                    if (tcnt != 0 && tpre < g.max_report) {
-                        const uint32_t k = atomicAdd(p.active_cnt, 1u);
-                        p.active[2 * k] = ((uint64_t)sgi << 40) | (t0 + tid);
-                        p.active[2 * k + 1] = tpre;
-                    }
-                }
-                if (tcnt != 0) tc[tid] = 0u;  // clean for the next call
-            }
-            __syncthreads();
-        }
-    }
-
-    grid_barrier(p.gbar, p.gbar_base);
-
-    // ------------------------------------------------------------ phase B
-    const uint32_t n_act = *(volatile uint32_t *)p.active_cnt;
     const uint64_t policy = evict_first_policy();
+    constexpr uint64_t kLtMask = (1ull << 40) - 1;
+
+    // re-read, re-evaluate and compact a list of active tiles {key, prefix}
     uint32_t phase[2] = {0u, 0u};
-    auto issue = [&](uint32_t k, int st) {
-        const uint64_t a = __ldcg(p.active + 2 * k);
-        const Seg &g = segs[a >> 40];
+    auto issue = [&](uint64_t key, int st) {
+        const Seg &g = segs[key >> 40];
         StageInfo si;
         uintptr_t ao, ar;
         uint32_t nbo, nbr;
-        plan_tile(g, a & ((1ull << 40) - 1), si, ao, nbo, ar, nbr);
+        plan_tile(g, key & kLtMask, si, ao, nbo, ar, nbr);
         uint8_t *dst = smem + (size_t)st * kStageBytes;
         mbar_arrive_expect_tx(&bar[st], nbo + nbr);
         bulk_g2s(dst, reinterpret_cast<const void *>(ao), nbo, &bar[st], policy);
         bulk_g2s(dst + kStageArrayBytes, reinterpret_cast<const void *>(ar), nbr, &bar[st], policy);
     };
-    ThreadAcc dummy;
-    dummy.reset();
-    int st = 0;
-    if (blockIdx.x < n_act && tid == 0) issue(blockIdx.x, 0);
-    for (uint32_t k = blockIdx.x; k < n_act; k += gridDim.x) {
-        const uint32_t nk = k + gridDim.x;
-        if (nk < n_act && tid == 0) issue(nk, st ^ 1);  // prefetch the next active tile
-        const uint64_t a = __ldcg(p.active + 2 * k);
-        const uint64_t excl = __ldcg(p.active + 2 * k + 1);
-        const Seg &g = segs[a >> 40];
-        StageInfo si;
-        uintptr_t ao, ar;
-        uint32_t nbo, nbr;
-        plan_tile(g, a & ((1ull << 40) - 1), si, ao, nbo, ar, nbr);
-        mbar_wait(&bar[st], phase[st]);
-        phase[st] ^= 1u;
-        const uint8_t *so = smem + (size_t)st * kStageBytes;
-        SegHot gh;
-        gh.load(g);
-        const uint64_t mask = eval_any(so, so + kStageArrayBytes, si, tid, gh, dummy);
-        compact_any(g, si, mask, excl, s_w);
-        __syncthreads();  // stage `st` and s_w are reused
-        st ^= 1;
+    auto process = [&](uint32_t n, auto get_key, auto get_pre) {
+        ThreadAcc dummy;
+        dummy.reset();
+        int st = 0;
+        if (n > 0 && tid == 0) issue(get_key(0u), 0);
+        for (uint32_t j = 0; j < n; ++j) {
+            if (j + 1 < n && tid == 0) issue(get_key(j + 1), st ^ 1);  // prefetch the next tile
+            const uint64_t key = get_key(j);
+            const uint64_t excl = get_pre(j);
+            const Seg &g = segs[key >> 40];
+            StageInfo si;
+            uintptr_t ao, ar;
+            uint32_t nbo, nbr;
+            plan_tile(g, key & kLtMask, si, ao, nbo, ar, nbr);
+            mbar_wait(&bar[st], phase[st]);
+            phase[st] ^= 1u;
+            const uint8_t *so = smem + (size_t)st * kStageBytes;
+            SegHot gh;
+            gh.load(g);
+            const uint64_t mask = eval_any(so, so + kStageArrayBytes, si, tid, gh, dummy);
+            compact_any(g, si, mask, excl, s_w);
+            __syncthreads();  // stage `st` and s_w are reused
+            st ^= 1;
+        }
+    };
+
+    const uint32_t n_nz = *(volatile uint32_t *)p.nz_cnt;
+    if (n_nz <= (uint32_t)kPoolCap) {
+        // ------------------------------------------------------ pool path
+        // arrive on the grid-barrier counter without waiting: the host advances
+        // its base by gridDim.x for every launch
+        if (tid == 0) atomicAdd(p.gbar, 1ull);
+        for (uint32_t i = tid; i < n_nz; i += kConsumerThreads) {
+            s_pkey[i] = __ldcg(p.nz_list + 2 * i);
+            s_pcnt[i] = (uint32_t)__ldcg(p.nz_list + 2 * i + 1);
+        }
+        if (tid == 0) s_n = 0;
+        __syncthreads();
+        for (uint32_t k = blockIdx.x; k < n_nz; k += gridDim.x) {
+            const uint64_t key = s_pkey[k];
+            const uint64_t seg = key >> 40, lt = key & kLtMask;
+            uint64_t pre = 0, segtot = 0;
+            for (uint32_t i = tid; i < n_nz; i += kConsumerThreads) {
+                const uint64_t ki = s_pkey[i];
+                if ((ki >> 40) == seg) {
+                    segtot += s_pcnt[i];
+                    pre += ((ki & kLtMask) < lt) ? s_pcnt[i] : 0u;
+                }
+            }
+            uint64_t pre_tot, seg_tot;
+            block_excl_scan(pre, s_w, &pre_tot);
+            block_excl_scan(segtot, s_w, &seg_tot);
+            const Seg &g = segs[seg];
+            uint64_t base = 0;
+            if (g.flags & kSegBaseFromAcc) base = __ldcg(&p.acc[g.acc_slot].count) - seg_tot;
+            if (tid == 0) {
+                p.tile_cnt[g.slot_begin + lt] = 0u;  // clean for the next call
+                if (base + pre_tot < g.max_report && s_n < (uint32_t)kPoolLocal) {
+                    s_loc_key[s_n] = key;
+                    s_loc_pre[s_n] = base + pre_tot;
+                    s_n = s_n + 1;
+                }
+            }
+        }
+        __syncthreads();
+        const uint32_t n_loc = s_n;
+        process(n_loc, [&](uint32_t j) { return s_loc_key[j]; }, [&](uint32_t j) { return s_loc_pre[j]; });
+    } else {
+        // ------------------------------------------------------ group path
+        for (uint32_t sgi = 0; sgi < p.n_segs; ++sgi) {
+            const Seg &g = segs[sgi];
+            if (g.max_report == 0 || g.n == 0) continue;
+            const uint64_t ntiles = (g.n + tile_elems(g.dtype) - 1) / tile_elems(g.dtype);
+            const uint64_t ngroups = (ntiles + kGroupTiles - 1) / kGroupTiles;
+            const uint32_t *gc = p.group_cnt + g.group_begin;
+            uint64_t tot = 0;
+            for (uint64_t k = tid; k < ngroups; k += kConsumerThreads) tot += __ldcg(gc + k);
+            uint64_t total;
+            block_excl_scan(tot, s_w, &total);
+            if (total == 0) continue;  // uniform: nothing to report or to clear
+            uint64_t base = 0;
+            if (g.flags & kSegBaseFromAcc) base = __ldcg(&p.acc[g.acc_slot].count) - total;
+
+            uint64_t run = base, ord_run = 0;
+            for (uint64_t c0 = 0; c0 < ngroups; c0 += kGroupTiles) {
+                const uint64_t gi = c0 + tid;
+                const uint32_t cnt = gi < ngroups ? __ldcg(gc + gi) : 0u;
+                // pack (nonzero ordinal, count): group counts < 2^23, 256 of them < 2^31
+                const uint64_t v = ((uint64_t)(cnt != 0) << 40) | cnt;
+                uint64_t ctot;
+                const uint64_t ex = block_excl_scan(v, s_w, &ctot);
+                const uint64_t gpre = run + (ex & ((1ull << 40) - 1));
+                const uint64_t ord = ord_run + (ex >> 40);
+                if (tid == 0) s_n = 0;
+                __syncthreads();
+                if (cnt != 0 && (ord % gridDim.x) == blockIdx.x) {
+                    const uint32_t k = atomicAdd(&s_n, 1u);
+                    s_owned[k] = (uint32_t)gi;
+                    s_owned_pre[k] = gpre;
+                }
+                __syncthreads();
+                const uint32_t n_owned = s_n;
+                run += ctot & ((1ull << 40) - 1);
+                ord_run += ctot >> 40;
+                for (uint32_t q = 0; q < n_owned; ++q) {
+                    const uint64_t t0 = (uint64_t)s_owned[q] * kGroupTiles;
+                    const uint64_t gp = s_owned_pre[q];
+                    const uint64_t tg = ntiles - t0 < (uint64_t)kGroupTiles ? ntiles - t0 : (uint64_t)kGroupTiles;
+                    uint32_t *tc = p.tile_cnt + g.slot_begin + t0;
+                    const uint32_t tcnt = (uint64_t)tid < tg ? __ldcg(tc + tid) : 0u;
+                    if (gp < g.max_report) {  // uniform
+                        uint64_t gtot;
+                        const uint64_t tpre = gp + block_excl_scan(tcnt, s_w, &gtot);
+                        if (tcnt != 0 && tpre < g.max_report) {
+                            const uint32_t k = atomicAdd(p.active_cnt, 1u);
+                            p.active[2 * k] = ((uint64_t)sgi << 40) | (t0 + tid);
+                            p.active[2 * k + 1] = tpre;
+                        }
+                    }
+                    if (tcnt != 0) tc[tid] = 0u;  // clean for the next call
+                }
+                __syncthreads();
+            }
+        }
+        grid_barrier(p.gbar, p.gbar_base);
+        const uint32_t n_act = *(volatile uint32_t *)p.active_cnt;
+        const uint32_t mine = n_act > blockIdx.x ? (n_act - blockIdx.x + gridDim.x - 1) / gridDim.x : 0u;
+        process(mine, [&](uint32_t j) { return __ldcg(p.active + 2 * (blockIdx.x + j * gridDim.x)); },
+                [&](uint32_t j) { return __ldcg(p.active + 2 * (blockIdx.x + j * gridDim.x) + 1); });
     }
     if (p.finalize) finalize_launch(p, tid, kConsumerThreads, &s_last);
 }

@@ -114,6 +114,23 @@ PtrKind classify(const void *p, int device) {
     }
 }
 
+constexpr int kCompactSmem = 2 * kStageBytes + kPoolCap * (8 + 4);
+
+// Pinned host reports up to this many entries are written by the kernel over
+// PCIe; larger ones are staged in HBM and copied with one bulk D2H.
+constexpr uint64_t kDirectReportMax = 1 << 16;
+
+// Device alias of page-locked host memory (cudaMallocHost / cudaHostRegister /
+// torch pin_memory), or NULL.  Kernels write small results there directly.
+static void *pinned_device_alias(const void *p) {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return nullptr;
+    }
+    return a.type == cudaMemoryTypeHost ? a.devicePointer : nullptr;
+}
+
 int validate_region(const void *out, const void *ref, uint64_t n, int dtype, double abs_tol, double rel_tol,
                     uint64_t max_report, const arc_verify_result_t *res) {
     if (!res) { set_error("result is NULL"); return ARC_E_INVAL; }
@@ -223,6 +240,9 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
     p.active = c.active;
     p.active_cnt = c.active_cnt + c.parity;
     p.active_cnt_zero = c.active_cnt + (c.parity ^ 1);
+    p.nz_list = c.nz_list;
+    p.nz_cnt = c.nz_cnt + c.parity;
+    p.nz_cnt_zero = c.nz_cnt + (c.parity ^ 1);
     p.gbar = c.counters + 2;
     p.gbar_base = c.gbar_base;
     p.acc = c.acc + acc_lo;
@@ -247,7 +267,7 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
         const uint32_t grid2 = (uint32_t)c.num_sms;
         void *args[] = {&p};
         e = cudaLaunchCooperativeKernel((const void *)arcv_compact_kernel, dim3(grid2), dim3(kConsumerThreads), args,
-                                        2 * kStageBytes, c.stream);
+                                        kCompactSmem, c.stream);
         if (e != cudaSuccess) return cuda_fail(e, "arcv_compact_kernel cooperative launch");
         c.launches++;
         c.gbar_base += grid2;
@@ -280,9 +300,26 @@ static int begin_call(Ctx &c, uint64_t tile_slots, uint32_t n_acc) {
     if (st) return st;
     st = grow_device(&c.acc, &c.acc_cap, std::max<uint32_t>(n_acc, 1), true, c.stream);
     if (st) return st;
-    st = grow_device(&c.result_dev, &c.result_dev_cap, std::max<uint32_t>(n_acc, 1), false, c.stream);
-    if (st) return st;
-    return grow_pinned(&c.result_host, &c.result_host_cap, std::max<uint32_t>(n_acc, 1));
+    // result slots live in mapped pinned host memory: the last CTA writes them
+    // over PCIe, so a call needs no D2H copy, only one stream sync.
+    if (c.result_host_cap < std::max<uint32_t>(n_acc, 1)) {
+        if (c.result_host) {
+            CK(cudaStreamSynchronize(c.stream));
+            CK(cudaFreeHost(c.result_host));
+        }
+        c.result_host = nullptr;
+        c.result_host_cap = 0;
+        const size_t cap = std::max<size_t>(std::max<uint32_t>(n_acc, 1), 64);
+        cudaError_t e = cudaHostAlloc(reinterpret_cast<void **>(&c.result_host), cap * sizeof(Acc), cudaHostAllocMapped);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            set_error("cudaHostAlloc(result slots) failed: %s", cudaGetErrorString(e));
+            return ARC_E_NOMEM;
+        }
+        CK(cudaHostGetDevicePointer(reinterpret_cast<void **>(&c.result_dev), c.result_host, 0));
+        c.result_host_cap = cap;
+    }
+    return ARC_OK;
 }
 
 // Stream one region whose out and/or ref live in host memory through the chunk
@@ -375,6 +412,8 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
                 pl.dreport = dev_reports[k];
             } else if (classify(results[k].report, c.device) == PK_DEVICE) {
                 pl.dreport = results[k].report;
+            } else if (void *alias = cap <= kDirectReportMax ? pinned_device_alias(results[k].report) : nullptr) {
+                pl.dreport = static_cast<arc_mismatch_t *>(alias);  // small pinned report: written over PCIe by K2
             } else {
                 pl.host_report = true;
                 pl.stage_off = stage_entries;
@@ -419,10 +458,7 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
         if (st) return st;
     }
     const uint32_t n_slots = next_slot;
-    if (n_slots) {
-        CK(cudaMemcpyAsync(c.result_host, c.result_dev, n_slots * sizeof(Acc), cudaMemcpyDeviceToHost, c.stream));
-        CK(cudaStreamSynchronize(c.stream));
-    }
+    if (n_slots) CK(cudaStreamSynchronize(c.stream));  // result slots are mapped host memory
     if (c.timing) {
         st = collect_timing(c);
         if (st) return st;
@@ -488,6 +524,8 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
     if (opts) o = *opts;
     if (o.nranks < 1 || o.rank < 0 || o.rank >= o.nranks) { set_error("bad rank/nranks"); return ARC_E_INVAL; }
     if (o.nranks > 1 && !o.nccl_unique_id) { set_error("nranks > 1 needs nccl_unique_id"); return ARC_E_INVAL; }
+    // an NCCL id selects the collective path even for one rank (a 1-rank
+    // communicator), which lets a single GPU exercise it end to end
     int ndev = 0;
     cudaError_t e = cudaGetDeviceCount(&ndev);
     if (e != cudaSuccess) { cudaGetLastError(); return cuda_fail(e, "cudaGetDeviceCount"); }
@@ -504,6 +542,11 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
     c->rank = o.rank;
     c->nranks = o.nranks;
     c->num_sms = prop.multiProcessorCount;
+    if (c->num_sms * kPoolLocal < kPoolCap) {  // K2 pool path: per-CTA share must fit
+        set_error("device has %d SMs; need >= %d", c->num_sms, kPoolCap / kPoolLocal);
+        delete c;
+        return ARC_E_UNSUPPORTED;
+    }
     if (o.stream) {
         c->stream = static_cast<cudaStream_t>(o.stream);
         c->own_stream = false;
@@ -526,20 +569,25 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
     const size_t smem = (size_t)c->stages * kStageBytes;
     KernelFn kf = stream_kernel_for(c->stages);
     CK(cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    CK(cudaFuncSetAttribute(arcv_compact_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * kStageBytes));
+    CK(cudaFuncSetAttribute(arcv_compact_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kCompactSmem));
     int occ = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kf, kThreads, smem));
     if (occ < 1) { set_error("kernel does not fit on an SM (smem %zu)", smem); return ARC_E_UNSUPPORTED; }
     const int cap = env_int("ARCV_CTAS_PER_SM", 0);
     c->ctas_per_sm = cap > 0 ? std::min(cap, occ) : occ;
-    // counters: [0] tile tickets, [1] finished CTAs, [2] K2 grid barrier, then 2 x u32 active counts
-    e = cudaMalloc(&c->counters, 4 * sizeof(unsigned long long));
+    // counters: [0] tile tickets, [1] finished CTAs, [2] K2 grid barrier,
+    // [3] 2 x u32 active-list lengths, [4] 2 x u32 pool lengths (by parity)
+    e = cudaMalloc(&c->counters, 8 * sizeof(unsigned long long));
     if (e != cudaSuccess) { cudaGetLastError(); set_error("cudaMalloc counters"); return ARC_E_NOMEM; }
-    CK(cudaMemsetAsync(c->counters, 0, 4 * sizeof(unsigned long long), c->stream));
+    CK(cudaMemsetAsync(c->counters, 0, 8 * sizeof(unsigned long long), c->stream));
     c->active_cnt = reinterpret_cast<uint32_t *>(c->counters + 3);
+    c->nz_cnt = reinterpret_cast<uint32_t *>(c->counters + 4);
+    e = cudaMalloc(&c->nz_list, 2 * kPoolCap * sizeof(uint64_t));
+    if (e != cudaSuccess) { cudaGetLastError(); set_error("cudaMalloc pool list"); return ARC_E_NOMEM; }
     CK(cudaStreamSynchronize(c->stream));
     g_ctx = c;
-    if (o.nranks > 1) {
+    c->sharded = o.nccl_unique_id != nullptr;
+    if (c->sharded) {
         int st = shard_init(*c, o.nccl_unique_id);
         if (st) {
             arc_verify_finalize();
@@ -557,14 +605,14 @@ int arc_verify_finalize(void) {
     cudaFree(c->counters);
     cudaFree(c->tile_cnt);
     cudaFree(c->active);
+    cudaFree(c->nz_list);
     cudaFree(c->group_cnt);
     cudaFree(c->acc);
-    cudaFree(c->result_dev);
     cudaFree(c->seg_dev);
     cudaFree(c->report_stage);
     cudaFree(c->packet);
     cudaFree(c->gathered);
-    if (c->result_host) cudaFreeHost(c->result_host);
+    if (c->result_host) cudaFreeHost(c->result_host);  // result_dev is its device alias
     if (c->seg_host) cudaFreeHost(c->seg_host);
     if (c->hdr_host) cudaFreeHost(c->hdr_host);
     for (int b = 0; b < Ctx::kNBuf; ++b) {
@@ -624,7 +672,7 @@ int arc_verify_compare(const void *out, const void *ref, uint64_t n, arc_dtype_t
     r.rel_tol = rel_tol;
     r.max_report = max_report;
     r.name = nullptr;
-    if (g_ctx->nranks > 1) return shard_compare(*g_ctx, r, result);
+    if (g_ctx->sharded) return shard_compare(*g_ctx, r, result);
     return run_local(*g_ctx, &r, 1, result, nullptr, true, nullptr);
 }
 

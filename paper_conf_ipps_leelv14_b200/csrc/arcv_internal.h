@@ -18,6 +18,7 @@ struct Ctx {
 
     int device = 0;
     int rank = 0, nranks = 1;
+    bool sharded = false;  // collective path (NCCL communicator), nranks >= 1
     int num_sms = 0, ctas_per_sm = 1, stages = 3, flags = 0;
     cudaStream_t stream = nullptr;
     bool own_stream = false;
@@ -31,12 +32,14 @@ struct Ctx {
     uint32_t *tile_cnt = nullptr;      size_t tile_cnt_cap = 0;   // per-tile counts (kept zero)
     uint64_t *active = nullptr;        size_t active_cap = 0;     // K2 active list (2 words / entry)
     uint32_t *active_cnt = nullptr;                               // [2] by parity
+    uint64_t *nz_list = nullptr;                                  // K1 -> K2 pool (kPoolCap entries)
+    uint32_t *nz_cnt = nullptr;                                   // [2] by parity
     unsigned long long gbar_base = 0;
     uint32_t *group_cnt = nullptr;     size_t group_cap = 0;      // [2][group_cap], parity per K1
     int parity = 0;
     Acc *acc = nullptr;                size_t acc_cap = 0;
-    Acc *result_dev = nullptr;         size_t result_dev_cap = 0;
-    Acc *result_host = nullptr;        size_t result_host_cap = 0;
+    Acc *result_host = nullptr;        size_t result_host_cap = 0;   // mapped pinned
+    Acc *result_dev = nullptr;                                       // its device alias
     Seg *seg_dev = nullptr;            size_t seg_dev_cap = 0;
     Seg *seg_host = nullptr;           size_t seg_host_cap = 0;
     arc_mismatch_t *report_stage = nullptr; size_t report_stage_cap = 0;

@@ -16,6 +16,8 @@ constexpr int kThreads = kConsumerThreads + 32;     // + producer warp
 constexpr int kVecPerThread = kTileBytes / 16 / kConsumerThreads;  // 4
 constexpr int kMaxInlineSegs = 8;
 constexpr int kGroupTiles = 256;                    // tiles per group counter
+constexpr int kPoolCap = 2048;                      // K2 pool path: max listed nonzero tiles
+constexpr int kPoolLocal = 64;                      // per-CTA share of the pool (grid >= 32)
 static_assert(kVecPerThread == 4, "packed-scan layout assumes 4 vectors per thread");
 static_assert(kGroupTiles == kConsumerThreads, "K2 scans one group per block pass");
 
@@ -64,7 +66,10 @@ struct Params {
     uint64_t n_group_zero;
     uint64_t *active;         // K2 active-tile list: {seg << 40 | tile, prefix}
     uint32_t *active_cnt;     // this launch's list length
-    uint32_t *active_cnt_zero;  // the other parity, zeroed by K2 for the next launch
+    uint32_t *active_cnt_zero;  // the other parity, zeroed by K1 for the next launch
+    uint64_t *nz_list;        // K1 -> K2 pool: {seg << 40 | tile, count} of nonzero tiles
+    uint32_t *nz_cnt;         // this launch's pool length (may exceed kPoolCap: overflow)
+    uint32_t *nz_cnt_zero;    // the other parity
     unsigned long long *gbar; // K2 grid barrier counter (monotonic)
     unsigned long long gbar_base;
     Acc *acc;

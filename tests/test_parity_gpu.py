@@ -395,3 +395,65 @@ def test_prefilter_ulp_sweep(av, orc):
     for at, rt in [(1e-6, 1e-5), (0.0, 1e-5), (0.0, 1.2e-7), (1e-40, 0.0)]:
         run_both(av, orc, torch.from_numpy(out).cuda(), torch.from_numpy(ref).cuda(), "f32", at, rt, 100000,
                  f"ulp sweep {at} {rt}")
+
+
+@pytest.mark.parametrize("mr", [100, (1 << 16) + 1])
+def test_pinned_report(av, orc, mr):
+    """Pinned host report buffers: small ones are written by the kernel over PCIe,
+    large ones staged; both must equal the oracle."""
+    o5, r5 = synth.C5(1 << 20).slice(device="cuda")
+    rep = torch.empty(24 * mr, dtype=torch.uint8, pin_memory=True).numpy().view(av.REPORT_DTYPE)
+    g = av.compare(o5, r5, 0, 0, mr, report=rep)
+    o = orc.compare(o5.cpu().numpy(), r5.cpu().numpy(), "i32", 0, 0, mr)
+    assert_same(g, o, f"pinned mr={mr}")
+
+
+@pytest.mark.parametrize("n", [1, 15, 16, 17, 16384 * 3 + 5, (1 << 22) + 3])
+def test_u8_simd_path(av, orc, n):
+    gen = torch.Generator().manual_seed(n)
+    ref = torch.randint(0, 256, (n + 5,), generator=gen, dtype=torch.int32).to(torch.uint8)
+    out = ref.clone()
+    m = torch.rand(n + 5, generator=gen) < 0.003
+    out[m] = torch.randint(0, 256, (int(m.sum()),), generator=gen, dtype=torch.int32).to(torch.uint8)
+    for off in (0, 3):
+        o, r = out.cuda()[off:off + n], ref.cuda()[off:off + n]
+        run_both(av, orc, o, r, "u8", 0, 0, 1000, f"u8 n={n} off={off}")
+
+
+def test_collective_path_one_rank_nccl():
+    """The sharded/collective code path (NCCL all-gather + merge kernel + broadcast)
+    on a 1-rank communicator, in its own process (one library context per process)."""
+    import subprocess
+    import sys
+
+    script = os.path.join(os.path.dirname(__file__), "_nccl_one_rank.py")
+    res = subprocess.run([sys.executable, script], capture_output=True, text=True, timeout=600)
+    assert res.returncode == 0, res.stdout[-3000:] + res.stderr[-3000:]
+    assert "NCCL-ONE-RANK-OK" in res.stdout
+
+
+def test_host_streamed_dense_group_path(av, orc):
+    """Host-resident inputs with dense mismatches: chunked launches whose nonzero
+    tiles overflow K2's pool, so the group path runs with a per-chunk base."""
+    c5 = synth.C5(1 << 25)
+    out, ref = c5.slice()
+    mr = (1 << 24) + 7  # reaches into the second chunk
+    rep = np.zeros(mr, dtype=av.REPORT_DTYPE)
+    g = av.compare(out.pin_memory(), ref, 0, 0, mr, report=rep)
+    o = orc.compare(out.numpy(), ref.numpy(), "i32", 0, 0, mr)
+    assert_same(g, o, "host streamed dense")
+
+
+def test_pool_and_group_paths_alternate(av, orc):
+    """K2's sparse pool path and dense group path interleaved (shared counters,
+    grid-barrier bookkeeping) stay correct call after call."""
+    c1 = synth.C1()
+    o1, r1 = c1.slice()
+    o5, r5 = synth.C5(1 << 24).slice()  # 4096 nonzero tiles > pool capacity
+    e1 = orc.compare(o1.numpy(), r1.numpy(), "f32", 1e-6, 1e-5, 100)
+    e5 = orc.compare(o5.numpy(), r5.numpy(), "i32", 0, 0, 5000)
+    o1, r1, o5, r5 = o1.cuda(), r1.cuda(), o5.cuda(), r5.cuda()
+    for _ in range(6):
+        assert_same(av.compare(o1, r1, 1e-6, 1e-5, 100), e1, "pool")
+        assert_same(av.compare(o5, r5, 0, 0, 5000), e5, "group")
+        assert_same(av.compare(o1, r1, 1e-6, 1e-5, 100), e1, "pool again")
