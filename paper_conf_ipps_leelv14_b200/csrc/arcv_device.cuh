@@ -98,8 +98,9 @@ struct ThreadAcc {
     uint64_t count;
     double ma, rm;     // float dtypes: running max of d and r (fp64, exact)
     uint64_t imax;     // integer dtypes: running max |a - b|
+    bool seeded;       // float filter bounds seeded for this region
     __device__ void reset() {
-        count = 0; ma = 0.0; rm = 0.0; imax = 0;
+        count = 0; ma = 0.0; rm = 0.0; imax = 0; seeded = false;
     }
 };
 
@@ -108,12 +109,12 @@ struct ThreadAcc {
 struct SegHot {
     double abs_tol, rel_tol;
     uint64_t max_report, tile_begin, slot_begin, group_begin;
-    float rt_rd;
+    float at_rd, rt_rd;
     uint32_t dtype, acc_slot;
     __device__ __forceinline__ void load(const Seg &g) {
         abs_tol = g.abs_tol; rel_tol = g.rel_tol; max_report = g.max_report;
         tile_begin = g.tile_begin; slot_begin = g.slot_begin; group_begin = g.group_begin;
-        rt_rd = g.rt_rd; dtype = g.dtype; acc_slot = g.acc_slot;
+        at_rd = g.at_rd; rt_rd = g.rt_rd; dtype = g.dtype; acc_slot = g.acc_slot;
     }
 };
 
@@ -152,25 +153,40 @@ __device__ __forceinline__ bool eval_f64(double x, double y, double at, double r
 // Bounds only grow, so bounds read at the start of a tile are conservative.
 template <typename T>
 struct FastBounds {
-    T k, ma;
+    T k;      // min(rel_f, rm_f, 1/4)               (rel form)
+    T kr;     // min(rm_f, 1/4)                      (abs form)
+    T at;     // abs_f <= abs_tol                    (abs form)
+    T ma;     // RD_f(ma)
 };
 
-__device__ __forceinline__ void refresh_bounds(const ThreadAcc &acc, float rt_rd, FastBounds<float> &b) {
+__device__ __forceinline__ void refresh_bounds(const ThreadAcc &acc, float at_rd, float rt_rd,
+                                               FastBounds<float> &b) {
     b.ma = __double2float_rd(acc.ma);
-    b.k = fminf(fminf(rt_rd, __double2float_rd(__dmul_rd(acc.rm, 1.0 - 0x1p-40))), 0.25f);
+    b.kr = fminf(__double2float_rd(__dmul_rd(acc.rm, 1.0 - 0x1p-40)), 0.25f);
+    b.k = fminf(rt_rd, b.kr);
+    b.at = at_rd;
 }
-__device__ __forceinline__ void refresh_bounds(const ThreadAcc &acc, double rt, FastBounds<double> &b) {
+__device__ __forceinline__ void refresh_bounds(const ThreadAcc &acc, double at, double rt, FastBounds<double> &b) {
     b.ma = acc.ma;
-    b.k = fmin(fmin(rt, acc.rm), 0.25);
+    b.kr = fmin(acc.rm, 0.25);
+    b.k = fmin(rt, b.kr);
+    b.at = at;
 }
 
+// rel form (rel_tol > 0):  x == y  or  (d < RD(k|y|) and d <= ma_f)
+// abs form (rel_tol = 0):  x == y  or  (d < abs_f and d < RD(kr|y|) and d <= ma_f)
+// (kr <= 1/4 gives the Sterbenz exactness in both; abs_f <= abs_tol <= t.)
+template <bool kRel>
 __device__ __forceinline__ bool fast_ok(float x, float y, const FastBounds<float> &b) {
     const float d = fabsf(__fsub_rn(x, y));
-    return (x == y) | ((d < __fmul_rd(b.k, fabsf(y))) & (d <= b.ma));
+    if constexpr (kRel) return (x == y) | ((d < __fmul_rd(b.k, fabsf(y))) & (d <= b.ma));
+    else return (x == y) | ((d < b.at) & (d < __fmul_rd(b.kr, fabsf(y))) & (d <= b.ma));
 }
+template <bool kRel>
 __device__ __forceinline__ bool fast_ok(double x, double y, const FastBounds<double> &b) {
     const double d = fabs(__dsub_rn(x, y));
-    return (x == y) | ((d < __dmul_rd(b.k, fabs(y))) & (d <= b.ma));
+    if constexpr (kRel) return (x == y) | ((d < __dmul_rd(b.k, fabs(y))) & (d <= b.ma));
+    else return (x == y) | ((d < b.at) & (d < __dmul_rd(b.kr, fabs(y))) & (d <= b.ma));
 }
 
 template <typename T>
@@ -198,6 +214,39 @@ __device__ __forceinline__ uint64_t raw_bits(T v) {
     }
 }
 
+// Seed the running maxima once per region per thread: evaluate exactly the
+// thread's element with the largest |x - y| and the one with the largest
+// (approximate) |x - y| / |y| in its first tile, so that the fast pass starts
+// with near-final bounds instead of flagging every record-breaking element.
+// Evaluating an element here and again in the main pass is harmless: maxima
+// are idempotent and the mismatch decision is taken by the main pass.
+template <typename T>
+__device__ __forceinline__ void seed_bounds(const uint8_t *so, const uint8_t *sr, uint32_t off_o, uint32_t off_r,
+                                            uint32_t cnt, int ctid, const SegHot &g, ThreadAcc &acc) {
+    constexpr int EPV = 16 / sizeof(T);
+    acc.seeded = true;
+    float best_d = -1.f, best_r = -1.f;
+    int bd = -1, br = -1;
+    for (int b = 0; b < kVecPerThread * EPV; ++b) {
+        const uint32_t e = (uint32_t)(((b / EPV) * kConsumerThreads + ctid) * EPV + (b % EPV));
+        if (e >= cnt) continue;
+        const T x = *reinterpret_cast<const T *>(so + off_o + e * sizeof(T));
+        const T y = *reinterpret_cast<const T *>(sr + off_r + e * sizeof(T));
+        const float d = (float)fabs((double)x - (double)y);
+        const float r = __fdividef(d, fabsf((float)y) + 1e-37f);
+        if (d > best_d && d < CUDART_INF_F) { best_d = d; bd = b; }
+        if (r > best_r && r < CUDART_INF_F) { best_r = r; br = b; }
+    }
+    for (int q = 0; q < 2; ++q) {
+        const int b = q == 0 ? bd : br;
+        if (b < 0 || (q == 1 && br == bd)) continue;
+        const uint32_t e = (uint32_t)(((b / EPV) * kConsumerThreads + ctid) * EPV + (b % EPV));
+        const T x = *reinterpret_cast<const T *>(so + off_o + e * sizeof(T));
+        const T y = *reinterpret_cast<const T *>(sr + off_r + e * sizeof(T));
+        (void)eval_f64((double)x, (double)y, g.abs_tol, g.rel_tol, acc);
+    }
+}
+
 // Evaluate this thread's share of one tile; returns the mismatch bit mask
 // (bit k*EPV + j <-> tile element (k*256 + ctid)*EPV + j).  Floats: a fast pass
 // over all elements with the exact pre-filter, then the fp64 rule only for the
@@ -211,9 +260,16 @@ __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *
     uint32_t bmax = 0;  // u8 only: byte-wise running max |a - b|
     using RT = typename std::conditional<std::is_same<T, float>::value, float, double>::type;
     FastBounds<RT> fb;
+    bool rel_form = true;
     if constexpr (kFloat) {
-        if constexpr (std::is_same<T, float>::value) refresh_bounds(acc, g.rt_rd, fb);
-        else refresh_bounds(acc, g.rel_tol, fb);
+        if (!acc.seeded) seed_bounds<T>(so, sr, off_o, off_r, cnt, ctid, g, acc);
+        if constexpr (std::is_same<T, float>::value) {
+            refresh_bounds(acc, g.at_rd, g.rt_rd, fb);
+            rel_form = g.rt_rd > 0.f;
+        } else {
+            refresh_bounds(acc, g.abs_tol, g.rel_tol, fb);
+            rel_form = g.rel_tol > 0.0;
+        }
     }
 #pragma unroll
     for (int k = 0; k < kVecPerThread; ++k) {
@@ -256,8 +312,13 @@ __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *
             mask |= (uint64_t)(m16 & valid) << (k * EPV);
         } else if constexpr (kFloat) {
             uint32_t sl = 0;
+            if (rel_form) {
 #pragma unroll
-            for (int j = 0; j < EPV; ++j) sl |= (uint32_t)(!fast_ok((RT)xo[j], (RT)xr[j], fb)) << j;
+                for (int j = 0; j < EPV; ++j) sl |= (uint32_t)(!fast_ok<true>((RT)xo[j], (RT)xr[j], fb)) << j;
+            } else {
+#pragma unroll
+                for (int j = 0; j < EPV; ++j) sl |= (uint32_t)(!fast_ok<false>((RT)xo[j], (RT)xr[j], fb)) << j;
+            }
             slow |= (uint64_t)(sl & valid) << (k * EPV);
         } else {
             uint32_t mis = 0;
@@ -287,10 +348,10 @@ __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *
                 const T y = *reinterpret_cast<const T *>(sr + off_r + e * sizeof(T));
                 // the bounds grew since the fast pass: a re-check clears most of a
                 // warm-up tile's flags without the fp64 rule
-                if (fast_ok((RT)x, (RT)y, fb)) continue;
+                if (rel_form ? fast_ok<true>((RT)x, (RT)y, fb) : fast_ok<false>((RT)x, (RT)y, fb)) continue;
                 mask |= (uint64_t)eval_f64((double)x, (double)y, at, rt, acc) << b;
-                if constexpr (std::is_same<T, float>::value) refresh_bounds(acc, g.rt_rd, fb);
-                else refresh_bounds(acc, g.rel_tol, fb);
+                if constexpr (std::is_same<T, float>::value) refresh_bounds(acc, g.at_rd, g.rt_rd, fb);
+                else refresh_bounds(acc, g.abs_tol, g.rel_tol, fb);
             }
         }
     }
