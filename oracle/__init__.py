@@ -70,6 +70,13 @@ def _load():
             ctypes.c_double, ctypes.c_double, ctypes.c_uint64,
             ctypes.c_void_p, ctypes.POINTER(_Result),
         ]
+        lib.oracle_compare_ex.restype = ctypes.c_int
+        lib.oracle_compare_ex.argtypes = [
+            ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int,
+            ctypes.c_double, ctypes.c_double, ctypes.c_uint64,
+            ctypes.c_int, ctypes.c_double, ctypes.c_double, ctypes.c_double,
+            ctypes.c_void_p, ctypes.POINTER(_Result),
+        ]
         lib.oracle_sizeof_result.restype = ctypes.c_size_t
         lib.oracle_sizeof_mismatch.restype = ctypes.c_size_t
         assert lib.oracle_sizeof_result() == ctypes.sizeof(_Result)
@@ -95,8 +102,13 @@ class OracleError(ValueError):
     pass
 
 
-def compare(out, ref, dtype: str, abs_tol: float, rel_tol: float, max_report: int) -> OracleResult:
-    """Run the sequential oracle on two host arrays (numpy, contiguous)."""
+def compare(out, ref, dtype: str, abs_tol: float, rel_tol: float, max_report: int,
+            min_value=None, bounds=None) -> OracleResult:
+    """Run the sequential oracle on two host arrays (numpy, contiguous).
+
+    ``min_value`` (minValueToCheck, P:199) and ``bounds`` = (lo, hi) (value-bound
+    directives) select oracle_compare_ex (NEXT row N2).
+    """
     lib = _load()
     npdt = NP_DTYPES[dtype]
     out = np.ascontiguousarray(out, dtype=npdt).reshape(-1)
@@ -107,11 +119,21 @@ def compare(out, ref, dtype: str, abs_tol: float, rel_tol: float, max_report: in
     cap = min(int(max_report), n)
     report = np.zeros(max(cap, 1), dtype=REPORT_DTYPE)
     res = _Result()
-    st = lib.oracle_compare(
-        out.ctypes.data if n else None, ref.ctypes.data if n else None, n, DTYPES[dtype],
-        float(abs_tol), float(rel_tol), int(max_report),
-        report.ctypes.data if max_report > 0 else None, ctypes.byref(res),
-    )
+    if min_value is None and bounds is None:
+        st = lib.oracle_compare(
+            out.ctypes.data if n else None, ref.ctypes.data if n else None, n, DTYPES[dtype],
+            float(abs_tol), float(rel_tol), int(max_report),
+            report.ctypes.data if max_report > 0 else None, ctypes.byref(res),
+        )
+    else:
+        flags = (1 if min_value is not None else 0) | (2 if bounds is not None else 0)
+        lo, hi = bounds if bounds is not None else (0.0, 0.0)
+        st = lib.oracle_compare_ex(
+            out.ctypes.data if n else None, ref.ctypes.data if n else None, n, DTYPES[dtype],
+            float(abs_tol), float(rel_tol), int(max_report),
+            flags, float(min_value if min_value is not None else 0.0), float(lo), float(hi),
+            report.ctypes.data if max_report > 0 else None, ctypes.byref(res),
+        )
     if st != 0:
         raise OracleError("oracle_compare rejected its arguments")
     return OracleResult(int(res.n), int(res.n_mismatch), float(res.max_abs_err),

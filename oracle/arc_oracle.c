@@ -219,6 +219,91 @@ int oracle_compare(const void *out, const void *ref, uint64_t n, int dtype,
     return 0;
 }
 
+/*
+ * oracle_compare_ex -- the same definition with the two optional checks of
+ * sec. III-A / III-C (NEXT row N2; readings R10, R11 in DESIGN.md sec. 3):
+ *   check_flags & 1 (minValueToCheck: "result is compared only if its value
+ *       is bigger than a specified threshold"): element i is not compared when
+ *       |ref[i]| <= min_value -- it is a match and its d, r are excluded.  (A NaN
+ *       ref is compared: NaN <= t is false.)
+ *   check_flags & 2 (value bounds: "if they fall within the user-specified
+ *       bound, the tools will ignore the difference"): a mismatch with
+ *       lo <= out[i] <= hi is ignored -- it is a match and its d, r are excluded.
+ * Integer values enter both checks as (double) value, rounded to nearest.
+ */
+int oracle_compare_ex(const void *out, const void *ref, uint64_t n, int dtype,
+                      double abs_tol, double rel_tol, uint64_t max_report,
+                      int check_flags, double min_value, double lo, double hi,
+                      oracle_mismatch_t *report, oracle_result_t *res)
+{
+    uint64_t i;
+    int is_float;
+    double max_abs = 0.0, max_rel = 0.0;
+
+    if (res == NULL) return -1;
+    if (dtype < ORC_F32 || dtype > ORC_U8) return -1;
+    if (!(abs_tol >= 0.0) || !(rel_tol >= 0.0) || isinf(abs_tol) || isinf(rel_tol)) return -1;
+    if (n > 0 && (out == NULL || ref == NULL)) return -1;
+    if (max_report > 0 && report == NULL) return -1;
+    if ((check_flags & 1) && isnan(min_value)) return -1;
+    if ((check_flags & 2) && (isnan(lo) || isnan(hi))) return -1;
+
+    is_float = (dtype == ORC_F32 || dtype == ORC_F64);
+    res->n = n;
+    res->n_mismatch = 0;
+    res->n_reported = 0;
+
+    for (i = 0; i < n; ++i) {
+        int mismatch, has_d = 0, has_r = 0;
+        double d = 0.0, r = 0.0, xv, yv;
+        if (is_float) {
+            xv = load_float(out, dtype, i);
+            yv = load_float(ref, dtype, i);
+        } else if (dtype == ORC_I32) {
+            int32_t a, b;
+            memcpy(&a, (const char *)out + 4 * i, 4);
+            memcpy(&b, (const char *)ref + 4 * i, 4);
+            xv = (double)a; yv = (double)b;
+        } else if (dtype == ORC_I64) {
+            int64_t a, b;
+            memcpy(&a, (const char *)out + 8 * i, 8);
+            memcpy(&b, (const char *)ref + 8 * i, 8);
+            xv = (double)a; yv = (double)b;
+        } else {
+            xv = (double)((const uint8_t *)out)[i];
+            yv = (double)((const uint8_t *)ref)[i];
+        }
+        /* check 1: not compared */
+        if ((check_flags & 1) && fabs(yv) <= min_value)
+            continue;
+        if (is_float) {
+            mismatch = float_element(xv, yv, abs_tol, rel_tol, &has_d, &d, &has_r, &r);
+        } else {
+            uint64_t m = int_absdiff(out, ref, dtype, i);
+            d = (double)m;
+            has_d = 1;
+            mismatch = (m != 0);
+        }
+        /* check 2: an ignored difference */
+        if (mismatch && (check_flags & 2) && lo <= xv && xv <= hi)
+            continue;
+        if (has_d && d > max_abs) max_abs = d;
+        if (has_r && r > max_rel) max_rel = r;
+        if (mismatch) {
+            if (res->n_mismatch < max_report) {
+                report[res->n_mismatch].index = i;
+                report[res->n_mismatch].out_bits = raw_bits(out, dtype, i);
+                report[res->n_mismatch].ref_bits = raw_bits(ref, dtype, i);
+            }
+            res->n_mismatch += 1;
+        }
+    }
+    res->max_abs_err = max_abs;
+    res->max_rel_err = max_rel;
+    res->n_reported = res->n_mismatch < max_report ? res->n_mismatch : max_report;
+    return 0;
+}
+
 /* Size check for the ctypes binding. */
 size_t oracle_sizeof_result(void) { return sizeof(oracle_result_t); }
 size_t oracle_sizeof_mismatch(void) { return sizeof(oracle_mismatch_t); }

@@ -275,39 +275,46 @@ def _report_buffer(cap: int):
     return arr, arr.ctypes.data
 
 
+_RES = arc_verify_result_t()  # reused: one context per process, calls are serialised
+_compare_c = _lib.arc_verify_compare
+_RES_REF = ctypes.byref(_RES)
+
+
 def compare(out, ref, abs_tol: float = 0.0, rel_tol: float = 0.0, max_report: int = 1 << 20,
             report=None, n: Optional[int] = None) -> Result:
     """Verify ``out`` against ``ref`` (torch tensors, contiguous, same dtype).
 
     Tensors may live on the library's CUDA device or in (pinned) host memory.
-    ``report``: optional preallocated buffer -- a numpy REPORT_DTYPE array or a
-    CUDA uint8/int64 tensor of >= 24*cap bytes (then the report stays on the GPU).
+    ``report``: optional preallocated buffer -- a numpy REPORT_DTYPE array (pinned
+    if it comes from a pinned torch tensor) or a CUDA tensor of >= 24*cap bytes
+    (then the report stays on the GPU).
     """
-    if out.dtype != ref.dtype:
-        raise TypeError("out and ref dtypes differ")
-    if not (out.is_contiguous() and ref.is_contiguous()):
-        raise ValueError("tensors must be contiguous")
+    if _TORCH_CODES is None:
+        dtype_code(out)
+    code = _TORCH_CODES.get(out.dtype)
+    if code is None or out.dtype != ref.dtype:
+        raise TypeError(f"unsupported or mismatched dtypes {out.dtype} / {ref.dtype}")
     if n is None:
         n = out.numel()
         if ref.numel() != n:
             raise ValueError("size mismatch")
-    cap = min(int(max_report), n)
+    if n and not (out.is_contiguous() and ref.is_contiguous()):
+        raise ValueError("tensors must be contiguous")
     if report is None:
-        rep_arr, rep_ptr = _report_buffer(cap)
+        rep_arr, rep_ptr = _report_buffer(min(int(max_report), n))
     elif isinstance(report, np.ndarray):
         rep_arr, rep_ptr = report, report.ctypes.data
     else:
         rep_arr, rep_ptr = report, report.data_ptr()
-    res = arc_verify_result_t()
+    res = _RES
     res.report = rep_ptr if max_report > 0 else None
-    arc_verify_compare(out.data_ptr() if n else 0, ref.data_ptr() if n else 0, n, dtype_code(out),
-                       float(abs_tol), float(rel_tol), int(max_report), res)
-    if isinstance(rep_arr, np.ndarray):
-        rep = rep_arr[: res.n_reported]
-    else:
-        rep = rep_arr
-    return Result(int(res.n), int(res.n_mismatch), float(res.max_abs_err), float(res.max_rel_err),
-                  int(res.n_reported), rep)
+    st = _compare_c(out.data_ptr() if n else None, ref.data_ptr() if n else None, n, code,
+                    abs_tol, rel_tol, max_report, _RES_REF)
+    if st:
+        raise ArcVerifyError(st, "arc_verify_compare")
+    nr = res.n_reported
+    rep = rep_arr[:nr] if isinstance(rep_arr, np.ndarray) else rep_arr
+    return Result(res.n, res.n_mismatch, res.max_abs_err, res.max_rel_err, nr, rep)
 
 
 def batch(regions) -> list[Result]:

@@ -280,3 +280,60 @@ def test_generator_pinned_to_python():
     a = synth.C4().slice(1000, 5000)[0]
     b = synth.C4().slice(3000, 1000)[0]
     assert torch.equal(a[2000:3000].view(torch.int64), b.view(torch.int64))
+
+
+# ------------------------------------------------- N2: minValueToCheck / bounds
+def _numpy_expect_checks(out, ref, at, rt, min_value, bounds):
+    """Library-routine pin for the optional checks (readings R10, R11)."""
+    x = out.astype(np.float64)
+    y = ref.astype(np.float64)
+    with np.errstate(all="ignore"):
+        match = np.isclose(x, y, rtol=rt, atol=at, equal_nan=True)
+        d = np.where(x == y, 0.0, np.abs(x - y))
+        r = np.where(x == y, 0.0, np.where(np.isinf(y), np.inf, d / np.abs(y)))
+    keep = np.ones(x.size, dtype=bool)
+    if min_value is not None:
+        keep &= ~(np.abs(y) <= min_value)
+    if bounds is not None:
+        keep &= ~((~match) & (bounds[0] <= x) & (x <= bounds[1]))
+    mis = (~match) & keep
+    valid = keep & ~(np.isnan(x) | np.isnan(y))
+    dmax = float(np.max(d[valid])) if valid.any() else 0.0
+    rmax = float(np.max(r[valid])) if valid.any() else 0.0
+    return np.flatnonzero(mis), dmax, rmax
+
+
+@pytest.mark.parametrize("min_value,bounds", [(1e-32, None), (0.5, None), (None, (-0.25, 0.25)),
+                                              (1e-3, (0.0, 1.0)), (0.0, (-np.inf, np.inf))])
+def test_checks_vs_numpy(oracle_mod, min_value, bounds):
+    rng = np.random.default_rng(3)
+    out, ref = _boundary_pairs(rng, 100_003, "f32")
+    sp = np.array(synth.F32_SPECIAL_BITS, dtype=np.uint32).view(np.float32)
+    out = np.concatenate([out, np.repeat(sp, sp.size)])
+    ref = np.concatenate([ref, np.tile(sp, sp.size)])
+    idx, dmax, rmax = _numpy_expect_checks(out, ref, 1e-6, 1e-5, min_value, bounds)
+    res = oracle_mod.compare(out, ref, "f32", 1e-6, 1e-5, 10 ** 6, min_value=min_value, bounds=bounds)
+    assert res.n_mismatch == idx.size
+    assert np.array_equal(res.report["index"], idx.astype(np.uint64))
+    assert res.max_abs_err == dmax and res.max_rel_err == rmax
+
+
+def test_checks_hand_cases(oracle_mod):
+    """The paper's example minValueToCheck=1e-32 and a value bound."""
+    out = np.array([1e-40, 5e-33, 3.0, 0.6, np.nan], dtype=np.float64)
+    ref = np.array([0.0, 1e-33, 2.0, 0.5, 1.0], dtype=np.float64)
+    # without checks: 1e-40 vs 0 matches (abs 1e-6); 5e-33 vs 1e-33 matches; 3 vs 2, 0.6 vs 0.5, NaN vs 1 mismatch
+    r0 = oracle_mod.compare(out, ref, "f64", 1e-6, 1e-5, 10)
+    assert list(r0.report["index"]) == [2, 3, 4]
+    # minValueToCheck = 1e-32: elements 0, 1 are not compared (|ref| <= 1e-32): same mismatches,
+    # but max_rel no longer sees 1e-40/0 = inf
+    r1 = oracle_mod.compare(out, ref, "f64", 1e-6, 1e-5, 10, min_value=1e-32)
+    assert list(r1.report["index"]) == [2, 3, 4] and r1.max_rel_err == 0.5 and r0.max_rel_err == np.inf
+    # value bound [0, 1]: 0.6 vs 0.5 is ignored (out inside the bound), 3 vs 2 and NaN are not
+    r2 = oracle_mod.compare(out, ref, "f64", 1e-6, 1e-5, 10, bounds=(0.0, 1.0))
+    assert list(r2.report["index"]) == [2, 4] and r2.max_abs_err == 1.0
+    # integers enter the checks as doubles
+    a = np.array([5, 9, -3], dtype=np.int32)
+    b = np.array([0, 7, -3], dtype=np.int32)
+    r3 = oracle_mod.compare(a, b, "i32", 0, 0, 10, min_value=0.5)
+    assert list(r3.report["index"]) == [1] and r3.max_abs_err == 2.0
