@@ -103,6 +103,26 @@ typedef struct {
                                    path over a 1-rank communicator                        */
 } arc_verify_opts_t;
 
+/*
+ * Optional per-region checks (sec. III-A and III-C; NEXT row N2; DESIGN.md
+ * readings R10, R11).  flags = 0 disables both.
+ *   ARC_CHECK_MIN_VALUE  ("minValueToCheck": "result is compared only if
+ *       its value is bigger than a specified threshold"): element i is not
+ *       compared when |ref[i]| <= min_value -- it is a match and its d, r are
+ *       excluded from the maxima.  A NaN ref is still compared.
+ *   ARC_CHECK_VALUE_BOUNDS (value-bound directives: differences that "fall
+ *       within the user-specified bound" are ignored): a mismatch with
+ *       lo <= out[i] <= hi is ignored -- a match, d and r excluded.
+ * Integer values enter both checks as (double)value, rounded to nearest.
+ * Errors: ARC_E_INVAL for unknown flag bits or NaN min_value / lo / hi.
+ */
+enum { ARC_CHECK_MIN_VALUE = 1u, ARC_CHECK_VALUE_BOUNDS = 2u };
+typedef struct {
+    uint32_t flags;
+    double min_value;
+    double lo, hi;
+} arc_verify_check_t;
+
 typedef struct {
     const void *out;  /* region output computed by the GPU kernel                  */
     const void *ref;  /* sequential reference output                               */
@@ -111,6 +131,7 @@ typedef struct {
     double abs_tol, rel_tol;
     uint64_t max_report;
     const char *name; /* for printing only; may be NULL                            */
+    const arc_verify_check_t *check; /* optional checks (N2); NULL = none            */
 } arc_verify_region_t;
 
 /*
@@ -150,6 +171,15 @@ int arc_verify_init(const arc_verify_opts_t *opts);
 int arc_verify_compare(const void *out, const void *ref, uint64_t n, arc_dtype_t dtype,
                        double abs_tol, double rel_tol, uint64_t max_report,
                        arc_verify_result_t *result);
+
+/*
+ * arc_verify_compare_ex -- arc_verify_compare with the optional checks of
+ * arc_verify_check_t (check may be NULL).  Not collective in sharded mode
+ * unless check is NULL (the checks are then applied locally on each rank).
+ */
+int arc_verify_compare_ex(const void *out, const void *ref, uint64_t n, arc_dtype_t dtype,
+                          double abs_tol, double rel_tol, uint64_t max_report,
+                          const arc_verify_check_t *check, arc_verify_result_t *result);
 
 /*
  * arc_verify_batch -- verify n_regions regions ("all data written by the kernels

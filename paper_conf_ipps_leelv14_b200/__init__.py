@@ -37,7 +37,7 @@ EXPORTED = [
     "arc_verify_strerror", "arc_verify_last_error", "arc_verify_set_stream",
     "arc_verify_get_unique_id", "arc_verify_set_timing", "arc_verify_kernel_stats",
     "arc_verify_version", "arc_verify_merge_plan", "arc_verify_packet_bytes",
-    "arc_verify_shard_local", "arc_verify_shard_merge", "arc_verify_probe_read",
+    "arc_verify_shard_local", "arc_verify_shard_merge", "arc_verify_probe_read", "arc_verify_compare_ex",
 ]
 
 
@@ -58,10 +58,19 @@ class arc_verify_opts_t(ctypes.Structure):
                 ("nranks", ctypes.c_int), ("nccl_unique_id", ctypes.c_void_p)]
 
 
+ARC_CHECK_MIN_VALUE, ARC_CHECK_VALUE_BOUNDS = 1, 2
+
+
+class arc_verify_check_t(ctypes.Structure):
+    _fields_ = [("flags", ctypes.c_uint32), ("min_value", ctypes.c_double), ("lo", ctypes.c_double),
+                ("hi", ctypes.c_double)]
+
+
 class arc_verify_region_t(ctypes.Structure):
     _fields_ = [("out", ctypes.c_void_p), ("ref", ctypes.c_void_p), ("n", ctypes.c_uint64),
                 ("dtype", ctypes.c_int), ("abs_tol", ctypes.c_double), ("rel_tol", ctypes.c_double),
-                ("max_report", ctypes.c_uint64), ("name", ctypes.c_char_p)]
+                ("max_report", ctypes.c_uint64), ("name", ctypes.c_char_p),
+                ("check", ctypes.POINTER(arc_verify_check_t))]
 
 
 class arc_shard_header_t(ctypes.Structure):
@@ -102,6 +111,8 @@ def _load() -> ctypes.CDLL:
         "arc_verify_shard_local": (I, [P, P, U64, I, D, D, U64, P, U64]),
         "arc_verify_shard_merge": (I, [P, I, U64, U64, ctypes.POINTER(arc_verify_result_t)]),
         "arc_verify_probe_read": (I, [P, P, U64, I, ctypes.POINTER(D)]),
+        "arc_verify_compare_ex": (I, [P, P, U64, I, D, D, U64, ctypes.POINTER(arc_verify_check_t),
+                                      ctypes.POINTER(arc_verify_result_t)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -280,8 +291,22 @@ _compare_c = _lib.arc_verify_compare
 _RES_REF = ctypes.byref(_RES)
 
 
+def make_check(min_value: Optional[float] = None, bounds=None):
+    """arc_verify_check_t for minValueToCheck and/or value bounds (lo, hi)."""
+    if min_value is None and bounds is None:
+        return None
+    ck = arc_verify_check_t()
+    if min_value is not None:
+        ck.flags |= ARC_CHECK_MIN_VALUE
+        ck.min_value = float(min_value)
+    if bounds is not None:
+        ck.flags |= ARC_CHECK_VALUE_BOUNDS
+        ck.lo, ck.hi = float(bounds[0]), float(bounds[1])
+    return ck
+
+
 def compare(out, ref, abs_tol: float = 0.0, rel_tol: float = 0.0, max_report: int = 1 << 20,
-            report=None, n: Optional[int] = None) -> Result:
+            report=None, n: Optional[int] = None, min_value: Optional[float] = None, bounds=None) -> Result:
     """Verify ``out`` against ``ref`` (torch tensors, contiguous, same dtype).
 
     Tensors may live on the library's CUDA device or in (pinned) host memory.
@@ -308,8 +333,13 @@ def compare(out, ref, abs_tol: float = 0.0, rel_tol: float = 0.0, max_report: in
         rep_arr, rep_ptr = report, report.data_ptr()
     res = _RES
     res.report = rep_ptr if max_report > 0 else None
-    st = _compare_c(out.data_ptr() if n else None, ref.data_ptr() if n else None, n, code,
-                    abs_tol, rel_tol, max_report, _RES_REF)
+    ck = make_check(min_value, bounds)
+    if ck is None:
+        st = _compare_c(out.data_ptr() if n else None, ref.data_ptr() if n else None, n, code,
+                        abs_tol, rel_tol, max_report, _RES_REF)
+    else:
+        st = _lib.arc_verify_compare_ex(out.data_ptr() if n else None, ref.data_ptr() if n else None, n, code,
+                                        abs_tol, rel_tol, max_report, ctypes.byref(ck), _RES_REF)
     if st:
         raise ArcVerifyError(st, "arc_verify_compare")
     nr = res.n_reported
@@ -318,12 +348,13 @@ def compare(out, ref, abs_tol: float = 0.0, rel_tol: float = 0.0, max_report: in
 
 
 def batch(regions) -> list[Result]:
-    """regions: iterable of (out, ref, abs_tol, rel_tol, max_report[, name]) torch tensors."""
+    """regions: iterable of (out, ref, abs_tol, rel_tol, max_report[, name[, check]]) with torch
+    tensors; ``check`` is an arc_verify_check_t (see make_check) or None."""
     regions = list(regions)
     R = len(regions)
     regs = (arc_verify_region_t * R)()
     results = (arc_verify_result_t * R)()
-    keep = []
+    keep, keep_ck = [], []
     for k, reg in enumerate(regions):
         out, ref, at, rt, mr = reg[:5]
         name = reg[5] if len(reg) > 5 else None
@@ -334,8 +365,12 @@ def batch(regions) -> list[Result]:
         keep.append(arr)
         nm = name.encode() if name else None
         keep.append(nm)
+        ck = reg[6] if len(reg) > 6 else None
         regs[k] = arc_verify_region_t(out.data_ptr() if n else None, ref.data_ptr() if n else None, n,
-                                      dtype_code(out), float(at), float(rt), int(mr), nm)
+                                      dtype_code(out), float(at), float(rt), int(mr), nm,
+                                      ctypes.pointer(ck) if ck is not None else None)
+        if ck is not None:
+            keep_ck.append(ck)
         results[k].report = ptr if mr > 0 else None
     arc_verify_batch(regs, results)
     outs = []

@@ -110,11 +110,13 @@ struct SegHot {
     double abs_tol, rel_tol;
     uint64_t max_report, tile_begin, slot_begin, group_begin;
     float at_rd, rt_rd;
-    uint32_t dtype, acc_slot;
+    uint32_t dtype, acc_slot, cflags;
+    double minv, lo, hi;
     __device__ __forceinline__ void load(const Seg &g) {
         abs_tol = g.abs_tol; rel_tol = g.rel_tol; max_report = g.max_report;
         tile_begin = g.tile_begin; slot_begin = g.slot_begin; group_begin = g.group_begin;
         at_rd = g.at_rd; rt_rd = g.rt_rd; dtype = g.dtype; acc_slot = g.acc_slot;
+        cflags = g.cflags; minv = g.minv; lo = g.lo; hi = g.hi;
     }
 };
 
@@ -133,6 +135,21 @@ __device__ __forceinline__ bool eval_f64(double x, double y, double at, double r
         acc.rm = fmax(acc.rm, r);
     }
     return !match;
+}
+
+// eval_f64 with the optional N2 checks (arc_verify_check_t; readings R10/R11):
+// not compared when |ref| <= min_value; a mismatch with lo <= out <= hi is
+// ignored.  Either way: match, and d, r stay out of the maxima.
+__device__ __forceinline__ bool eval_f64_checked(double x, double y, const SegHot &g, ThreadAcc &acc) {
+    if (g.cflags == 0) return eval_f64(x, y, g.abs_tol, g.rel_tol, acc);
+    if ((g.cflags & ARC_CHECK_MIN_VALUE) && fabs(y) <= g.minv) return false;
+    if (g.cflags & ARC_CHECK_VALUE_BOUNDS) {
+        const double d = fabs(x - y);
+        const double t = __dadd_rn(g.abs_tol, __dmul_rn(g.rel_tol, fabs(y)));
+        const bool match = (x == y) | ((x != x) & (y != y)) | ((fabs(y) < CUDART_INF) & (d <= t));
+        if (!match && g.lo <= x && x <= g.hi) return false;
+    }
+    return eval_f64(x, y, g.abs_tol, g.rel_tol, acc);
 }
 
 // Exact pre-filter.  An element is finished without the
@@ -243,7 +260,7 @@ __device__ __forceinline__ void seed_bounds(const uint8_t *so, const uint8_t *sr
         const uint32_t e = (uint32_t)(((b / EPV) * kConsumerThreads + ctid) * EPV + (b % EPV));
         const T x = *reinterpret_cast<const T *>(so + off_o + e * sizeof(T));
         const T y = *reinterpret_cast<const T *>(sr + off_r + e * sizeof(T));
-        (void)eval_f64((double)x, (double)y, g.abs_tol, g.rel_tol, acc);
+        (void)eval_f64_checked((double)x, (double)y, g, acc);
     }
 }
 
@@ -292,7 +309,20 @@ __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *
             const uint32_t e0 = v * EPV;
             valid = e0 >= cnt ? 0u : (cnt - e0 >= (uint32_t)EPV ? valid : ((1u << (cnt - e0)) - 1u));
         }
-        if constexpr (std::is_same<T, uint8_t>::value) {
+        if (!kFloat && g.cflags != 0) {  // integers with N2 checks: plain scalar rule
+            uint32_t mis = 0;
+#pragma unroll
+            for (int j = 0; j < EPV; ++j) {
+                if (!((valid >> j) & 1u)) continue;
+                const double xv = (double)xo[j], yv = (double)xr[j];
+                if ((g.cflags & ARC_CHECK_MIN_VALUE) && fabs(yv) <= g.minv) continue;
+                const uint64_t m = int_absdiff<T>(xo[j], xr[j]);
+                if (m != 0 && (g.cflags & ARC_CHECK_VALUE_BOUNDS) && g.lo <= xv && xv <= g.hi) continue;
+                acc.imax = m > acc.imax ? m : acc.imax;
+                mis |= (uint32_t)(m != 0) << j;
+            }
+            mask |= (uint64_t)mis << (k * EPV);
+        } else if constexpr (std::is_same<T, uint8_t>::value) {
             // bytes: SIMD-within-a-register. |a-b| per byte (vabsdiffu4), running
             // byte-wise max (vmaxu4), and 4 mismatch bits per word from vcmpne4.
             uint32_t wa[4], wb[4], m16 = 0;
@@ -338,7 +368,6 @@ __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *
     }
     if constexpr (kFloat) {
         if (slow) {  // rare: mismatches, specials, new maxima
-            const double at = g.abs_tol, rt = g.rel_tol;
             uint64_t m = slow;
             while (m) {
                 const int b = __ffsll((long long)m) - 1;
@@ -349,7 +378,7 @@ __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *
                 // the bounds grew since the fast pass: a re-check clears most of a
                 // warm-up tile's flags without the fp64 rule
                 if (rel_form ? fast_ok<true>((RT)x, (RT)y, fb) : fast_ok<false>((RT)x, (RT)y, fb)) continue;
-                mask |= (uint64_t)eval_f64((double)x, (double)y, at, rt, acc) << b;
+                mask |= (uint64_t)eval_f64_checked((double)x, (double)y, g, acc) << b;
                 if constexpr (std::is_same<T, float>::value) refresh_bounds(acc, g.at_rd, g.rt_rd, fb);
                 else refresh_bounds(acc, g.abs_tol, g.rel_tol, fb);
             }

@@ -149,6 +149,20 @@ int validate_region(const void *out, const void *ref, uint64_t n, int dtype, dou
     return ARC_OK;
 }
 
+static int validate_check(const arc_verify_check_t *ck) {
+    if (!ck) return ARC_OK;
+    if (ck->flags & ~(uint32_t)(ARC_CHECK_MIN_VALUE | ARC_CHECK_VALUE_BOUNDS)) {
+        set_error("unknown check flags 0x%x", ck->flags);
+        return ARC_E_INVAL;
+    }
+    if (((ck->flags & ARC_CHECK_MIN_VALUE) && std::isnan(ck->min_value)) ||
+        ((ck->flags & ARC_CHECK_VALUE_BOUNDS) && (std::isnan(ck->lo) || std::isnan(ck->hi)))) {
+        set_error("check parameters must not be NaN");
+        return ARC_E_INVAL;
+    }
+    return ARC_OK;
+}
+
 // A float strictly below v (0 when v == 0): the fp32 pre-filter's tolerance
 // bounds (arcv_device.cuh eval_f32).
 static float lower_f32(double v) {
@@ -166,7 +180,7 @@ static uint64_t tiles_of(uint64_t n, uint32_t dtype) {
 
 static Seg make_seg(const void *out, const void *ref, uint64_t n, uint32_t dtype, double at, double rt,
                     uint64_t max_report, arc_mismatch_t *report, uint64_t slot_begin, uint64_t index_base,
-                    uint32_t acc_slot, uint32_t flags) {
+                    uint32_t acc_slot, uint32_t flags, const arc_verify_check_t *ck = nullptr) {
     Seg g;
     memset(&g, 0, sizeof(g));
     g.out = static_cast<const uint8_t *>(out);
@@ -183,6 +197,12 @@ static Seg make_seg(const void *out, const void *ref, uint64_t n, uint32_t dtype
     g.flags = flags;
     g.at_rd = lower_f32(at);
     g.rt_rd = lower_f32(rt);
+    if (ck && ck->flags) {
+        g.cflags = ck->flags;
+        g.minv = ck->min_value;
+        g.lo = ck->lo;
+        g.hi = ck->hi;
+    }
     return g;
 }
 
@@ -362,7 +382,7 @@ static int stream_region(Ctx &c, const arc_verify_region_t &r, bool out_dev, boo
         CK(cudaEventRecord(c.ev_copy[b], c.copy_stream));
         CK(cudaStreamWaitEvent(c.stream, c.ev_copy[b], 0));
         Seg g = make_seg(po, pr, ne, dtype, r.abs_tol, r.rel_tol, r.max_report, report, slot_base + e0 / te, e0, 0,
-                         kSegBaseFromAcc);
+                         kSegBaseFromAcc, r.check);
         int st = launch_segments(c, &g, 1, acc_slot, 1, ci + 1 == nchunks);
         if (st) return st;
         CK(cudaEventRecord(c.ev_free[b], c.stream));
@@ -388,6 +408,8 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
     for (size_t k = 0; k < R; ++k) {
         const arc_verify_region_t &r = regs[k];
         int st = validate_region(r.out, r.ref, r.n, r.dtype, r.abs_tol, r.rel_tol, r.max_report, &results[k]);
+        if (st) return st;
+        st = validate_check(r.check);
         if (st) return st;
         Plan &pl = plan[k];
         pl.out_dev = pl.ref_dev = true;
@@ -440,7 +462,7 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
         if (plan[k].stream || r.n == 0) continue;
         slot_of[k] = next_slot;
         segs.push_back(make_seg(r.out, r.ref, r.n, (uint32_t)r.dtype, r.abs_tol, r.rel_tol, r.max_report,
-                                plan[k].dreport, plan[k].slot_base, 0, next_slot, 0));
+                                plan[k].dreport, plan[k].slot_base, 0, next_slot, 0, r.check));
         next_slot++;
     }
     const uint32_t n_dev_slots = next_slot;
@@ -672,6 +694,25 @@ int arc_verify_compare(const void *out, const void *ref, uint64_t n, arc_dtype_t
     r.rel_tol = rel_tol;
     r.max_report = max_report;
     r.name = nullptr;
+    r.check = nullptr;
+    if (g_ctx->sharded) return shard_compare(*g_ctx, r, result);
+    return run_local(*g_ctx, &r, 1, result, nullptr, true, nullptr);
+}
+
+int arc_verify_compare_ex(const void *out, const void *ref, uint64_t n, arc_dtype_t dtype, double abs_tol,
+                          double rel_tol, uint64_t max_report, const arc_verify_check_t *check,
+                          arc_verify_result_t *result) {
+    if (!g_ctx) return ARC_E_NOINIT;
+    arc_verify_region_t r;
+    r.out = out;
+    r.ref = ref;
+    r.n = n;
+    r.dtype = dtype;
+    r.abs_tol = abs_tol;
+    r.rel_tol = rel_tol;
+    r.max_report = max_report;
+    r.name = nullptr;
+    r.check = (check && check->flags) ? check : nullptr;
     if (g_ctx->sharded) return shard_compare(*g_ctx, r, result);
     return run_local(*g_ctx, &r, 1, result, nullptr, true, nullptr);
 }

@@ -374,7 +374,7 @@ int arc_verify_shard_local(const void *out, const void *ref, uint64_t n, arc_dty
         set_error("packet must be device memory on the library's device");
         return ARC_E_INVAL;
     }
-    arc_verify_region_t r{out, ref, n, dtype, abs_tol, rel_tol, max_report, nullptr};
+    arc_verify_region_t r{out, ref, n, dtype, abs_tol, rel_tol, max_report, nullptr, nullptr};
     return local_packet(*g_ctx, r, static_cast<uint8_t *>(packet_dev));
 }
 

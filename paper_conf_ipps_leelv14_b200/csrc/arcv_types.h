@@ -41,7 +41,8 @@ struct Seg {
     uint32_t dtype;
     uint32_t flags;
     float at_rd, rt_rd;     // fp32 lower bounds of abs_tol / rel_tol (fp32 pre-filter)
-    uint32_t pad;
+    uint32_t cflags;        // ARC_CHECK_* (N2)
+    double minv, lo, hi;    // check parameters
 };
 
 struct Acc {  // per-region accumulators / result slot, 32 bytes

@@ -457,3 +457,43 @@ def test_pool_and_group_paths_alternate(av, orc):
         assert_same(av.compare(o1, r1, 1e-6, 1e-5, 100), e1, "pool")
         assert_same(av.compare(o5, r5, 0, 0, 5000), e5, "group")
         assert_same(av.compare(o1, r1, 1e-6, 1e-5, 100), e1, "pool again")
+
+
+# ---------------------------------------------- N2: minValueToCheck / bounds
+CHECKS = [(1e-32, None), (0.5, None), (None, (-0.25, 0.25)), (1e-3, (0.0, 1.0)), (0.0, (-np.inf, np.inf))]
+
+
+@pytest.mark.parametrize("dt", ["f32", "f64"])
+@pytest.mark.parametrize("mv,bounds", CHECKS)
+def test_checks_float(av, orc, dt, mv, bounds):
+    rng = np.random.default_rng(5)
+    out, ref = _boundary(rng, 1_000_003, dt)
+    sp = np.array(synth.F32_SPECIAL_BITS, dtype=np.uint32).view(np.float32).astype(NP[dt])
+    out = np.concatenate([out, np.repeat(sp, sp.size)])
+    ref = np.concatenate([ref, np.tile(sp, sp.size)])
+    o, r = torch.from_numpy(out).cuda(), torch.from_numpy(ref).cuda()
+    g = av.compare(o, r, 1e-6, 1e-5, 4000, min_value=mv, bounds=bounds)
+    e = orc.compare(out, ref, dt, 1e-6, 1e-5, 4000, min_value=mv, bounds=bounds)
+    assert_same(g, e, f"checks {dt} {mv} {bounds}")
+
+
+@pytest.mark.parametrize("dt", ["i32", "i64", "u8"])
+def test_checks_int(av, orc, dt):
+    o, r = random_pair(dt, 300_017, seed=9, rate=0.05)
+    for mv, bounds in [(3.0, None), (None, (0.0, 100.0)), (200.0, (10.0, 1e9))]:
+        g = av.compare(o, r, 0, 0, 1000, min_value=mv, bounds=bounds)
+        e = orc.compare(o.cpu().numpy(), r.cpu().numpy(), dt, 0, 0, 1000, min_value=mv, bounds=bounds)
+        assert_same(g, e, f"checks {dt} {mv} {bounds}")
+
+
+def test_checks_batch_and_streamed(av, orc):
+    c1 = synth.C1()
+    o, r = c1.slice()
+    ck = av.make_check(min_value=0.25, bounds=(-0.6, -0.4))
+    res = av.batch([(o.cuda(), r.cuda(), 1e-6, 1e-5, 100, "a", ck), (o.cuda(), r.cuda(), 1e-6, 1e-5, 100, "b")])
+    e_ck = orc.compare(o.numpy(), r.numpy(), "f32", 1e-6, 1e-5, 100, min_value=0.25, bounds=(-0.6, -0.4))
+    e = orc.compare(o.numpy(), r.numpy(), "f32", 1e-6, 1e-5, 100)
+    assert_same(res[0], e_ck, "batch checked")
+    assert_same(res[1], e, "batch plain")
+    g = av.compare(o.pin_memory(), r, 1e-6, 1e-5, 100, min_value=0.25, bounds=(-0.6, -0.4))
+    assert_same(g, e_ck, "host streamed checked")
