@@ -225,6 +225,50 @@ int arc_verify_kernel_stats(uint64_t *launches, double *total_ms, int reset);
  */
 int arc_verify_probe_read(const void *a, const void *b, uint64_t bytes, int iters, double *gbs);
 
+/*
+ * arc_verify_checksum -- the debug-assertion checksum screen (sec. III-C, P:291:
+ * "performing customized bug detection (e.g., establishing checksums and
+ * verifying them)"; NEXT row N4).  `data` is device memory on the library's
+ * device (any alignment), `bytes` its length.  out[0] = sum of h_i mod 2^64,
+ * out[1] = xor of h_i, where h_i = F(w_i + i * 0x9E3779B97F4A7C15), w_i the
+ * little-endian 64-bit words (last one zero-padded) and F the splitmix64
+ * finalizer.  Reads one array (half a comparison's bytes); equal checksums of a
+ * kernel output and of its reference mean bitwise-identical data with
+ * probability 1 - 2^-64 per pair.  Errors: ARC_E_INVAL, ARC_E_NOINIT, ARC_E_CUDA.
+ */
+int arc_verify_checksum(const void *data, uint64_t bytes, uint64_t out[2]);
+
+/* ------------------------------------------------------------------------
+ * Region selection and report printing (NEXT row N3), host-only.
+ * Sec. III-A: "a user can specify which specific kernels to verify by
+ * adding directives or using environment variables (e.g.,
+ * 'verificationOptions=complement=0,kernels=main_kernel0' ...)".  Reading
+ * (R20): comma-separated key=value pairs, an optional
+ * "verificationOptions=" prefix; `kernels` = region names separated by ':'
+ * (further comma tokens without '=' are also names); complement=0 (default)
+ * verifies only the listed regions, complement=1 all but them; no `kernels`
+ * key selects every region; other keys are ignored.  options == NULL reads the
+ * environment variable verificationOptions (then ARC_VERIFICATION_OPTIONS);
+ * unset selects every region.
+ * ------------------------------------------------------------------------ */
+
+/* 1 if region `name` is selected, 0 if not, ARC_E_INVAL for malformed options. */
+int arc_verify_selected(const char *options, const char *name);
+
+/* arc_verify_batch over the selected regions only; selected[k] (may be NULL)
+ * receives 1/0; an unselected region's result is zeroed (its report pointer
+ * kept).  Errors as arc_verify_batch, plus ARC_E_INVAL for malformed options. */
+int arc_verify_batch_selected(const arc_verify_region_t *regions, size_t n_regions, const char *options,
+                              arc_verify_result_t *results, uint8_t *selected);
+
+/* Human-readable report of one result ("an error will be reported to the user",
+ * P:199): a summary line, then up to max_entries entries "[index] out=.. ref=.."
+ * with decoded values and raw bits.  The report may be host or device memory.
+ * Writes a NUL-terminated string into buf (truncated to cap - 1 bytes) and
+ * returns the full length.  Errors: ARC_E_INVAL, ARC_E_CUDA. */
+int arc_verify_format_result(const char *name, arc_dtype_t dtype, double abs_tol, double rel_tol,
+                             const arc_verify_result_t *result, uint64_t max_entries, char *buf, size_t cap);
+
 /* ABI version (major << 16 | minor). */
 uint32_t arc_verify_version(void);
 

@@ -77,6 +77,8 @@ def _load():
             ctypes.c_int, ctypes.c_double, ctypes.c_double, ctypes.c_double,
             ctypes.c_void_p, ctypes.POINTER(_Result),
         ]
+        lib.oracle_checksum.restype = ctypes.c_int
+        lib.oracle_checksum.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.POINTER(ctypes.c_uint64)]
         lib.oracle_sizeof_result.restype = ctypes.c_size_t
         lib.oracle_sizeof_mismatch.restype = ctypes.c_size_t
         assert lib.oracle_sizeof_result() == ctypes.sizeof(_Result)
@@ -161,3 +163,13 @@ def merge_shards(parts, max_report: int) -> OracleResult:
     report = np.concatenate(entries) if entries else np.zeros(0, dtype=REPORT_DTYPE)
     n_rep = min(count, int(max_report))
     return OracleResult(n, count, max_abs, max_rel, n_rep, report[:n_rep].copy())
+
+
+def checksum(data) -> tuple[int, int]:
+    """The N4 debug-assertion checksum (sum, xor) of a host array's bytes."""
+    lib = _load()
+    b = np.ascontiguousarray(data).reshape(-1).view(np.uint8)
+    out = (ctypes.c_uint64 * 2)()
+    if lib.oracle_checksum(b.ctypes.data if b.size else None, b.size, out) != 0:
+        raise OracleError("oracle_checksum rejected its arguments")
+    return int(out[0]), int(out[1])

@@ -38,6 +38,7 @@ EXPORTED = [
     "arc_verify_get_unique_id", "arc_verify_set_timing", "arc_verify_kernel_stats",
     "arc_verify_version", "arc_verify_merge_plan", "arc_verify_packet_bytes",
     "arc_verify_shard_local", "arc_verify_shard_merge", "arc_verify_probe_read", "arc_verify_compare_ex",
+    "arc_verify_checksum", "arc_verify_selected", "arc_verify_batch_selected", "arc_verify_format_result",
 ]
 
 
@@ -113,6 +114,12 @@ def _load() -> ctypes.CDLL:
         "arc_verify_probe_read": (I, [P, P, U64, I, ctypes.POINTER(D)]),
         "arc_verify_compare_ex": (I, [P, P, U64, I, D, D, U64, ctypes.POINTER(arc_verify_check_t),
                                       ctypes.POINTER(arc_verify_result_t)]),
+        "arc_verify_checksum": (I, [P, U64, ctypes.POINTER(U64)]),
+        "arc_verify_selected": (I, [ctypes.c_char_p, ctypes.c_char_p]),
+        "arc_verify_batch_selected": (I, [ctypes.POINTER(arc_verify_region_t), SZ, ctypes.c_char_p,
+                                          ctypes.POINTER(arc_verify_result_t), P]),
+        "arc_verify_format_result": (I, [ctypes.c_char_p, I, D, D, ctypes.POINTER(arc_verify_result_t), U64,
+                                         ctypes.c_char_p, SZ]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -216,6 +223,48 @@ def arc_verify_probe_read(a_ptr: int, b_ptr: int, nbytes: int, iters: int = 10) 
     g = ctypes.c_double()
     _check(_lib.arc_verify_probe_read(a_ptr, b_ptr, nbytes, iters, ctypes.byref(g)), "arc_verify_probe_read")
     return float(g.value)
+
+
+def arc_verify_checksum(ptr: int, nbytes: int) -> tuple[int, int]:
+    out = (ctypes.c_uint64 * 2)()
+    _check(_lib.arc_verify_checksum(ptr or None, nbytes, out), "arc_verify_checksum")
+    return int(out[0]), int(out[1])
+
+
+def checksum(t) -> tuple[int, int]:
+    """Debug-assertion checksum (sum, xor) of a CUDA tensor's bytes (N4)."""
+    if not t.is_contiguous():
+        raise ValueError("tensor must be contiguous")
+    nb = t.numel() * t.element_size()
+    return arc_verify_checksum(t.data_ptr() if nb else 0, nb)
+
+
+def arc_verify_selected(options: Optional[str], name: str) -> bool:
+    st = _lib.arc_verify_selected(options.encode() if options is not None else None, name.encode())
+    if st < 0:
+        raise ArcVerifyError(st, "arc_verify_selected")
+    return bool(st)
+
+
+def arc_verify_format_result(name: str, dtype: int, abs_tol: float, rel_tol: float, result: arc_verify_result_t,
+                             max_entries: int = 10) -> str:
+    cap = 4096 + 256 * max_entries
+    buf = ctypes.create_string_buffer(cap)
+    st = _lib.arc_verify_format_result(name.encode() if name else None, dtype, abs_tol, rel_tol,
+                                       ctypes.byref(result), max_entries, buf, cap)
+    if st < 0:
+        raise ArcVerifyError(st, "arc_verify_format_result")
+    return buf.value.decode()
+
+
+def format_result(name: str, dtype: str, abs_tol: float, rel_tol: float, res: "Result",
+                  max_entries: int = 10) -> str:
+    """Report text for a Result (host numpy report) -- P:199 "reported to the user"."""
+    r = arc_verify_result_t(res.n, res.n_mismatch, res.max_abs_err, res.max_rel_err, res.n_reported, None)
+    rep = np.ascontiguousarray(res.report, dtype=REPORT_DTYPE) if res.n_reported else None
+    if rep is not None:
+        r.report = rep.ctypes.data
+    return arc_verify_format_result(name, DTYPE_CODES[dtype], abs_tol, rel_tol, r, max_entries)
 
 
 # ------------------------------------------------------------- conveniences
@@ -347,7 +396,7 @@ def compare(out, ref, abs_tol: float = 0.0, rel_tol: float = 0.0, max_report: in
     return Result(res.n, res.n_mismatch, res.max_abs_err, res.max_rel_err, nr, rep)
 
 
-def batch(regions) -> list[Result]:
+def batch(regions, options: Optional[str] = None, select: bool = False) -> list[Result]:
     """regions: iterable of (out, ref, abs_tol, rel_tol, max_report[, name[, check]]) with torch
     tensors; ``check`` is an arc_verify_check_t (see make_check) or None."""
     regions = list(regions)
@@ -372,7 +421,13 @@ def batch(regions) -> list[Result]:
         if ck is not None:
             keep_ck.append(ck)
         results[k].report = ptr if mr > 0 else None
-    arc_verify_batch(regs, results)
+    if select or options is not None:
+        sel = (ctypes.c_uint8 * R)()
+        st = _lib.arc_verify_batch_selected(regs, R, options.encode() if options is not None else None, results,
+                                            ctypes.cast(sel, ctypes.c_void_p))
+        _check(st, "arc_verify_batch_selected")
+    else:
+        arc_verify_batch(regs, results)
     outs = []
     for k in range(R):
         r = results[k]

@@ -1,0 +1,141 @@
+// arcv_checksum.cu -- NEXT row N4: the debug-assertion checksum screen.
+//
+// Sec. III-C: "we introduce a debug assertion API.  The users can
+// implement the API by performing customized bug detection (e.g., establishing
+// checksums and verifying them).  The API will be inserted at the end of the
+// kernel call."  This is a device checksum of ONE array (half the bytes of a
+// full comparison): comparing the checksum of a kernel's output with a stored
+// checksum of the reference screens for any bit change before a full compare.
+//
+// Definition (identical to oracle_checksum): little-endian
+// 64-bit words w_i (last one zero-padded), h_i = F(w_i + i*0x9E3779B97F4A7C15)
+// with F the splitmix64 finalizer; result = (sum h_i mod 2^64, xor h_i).  Both
+// reductions are order-independent, so any grid gives the same bits.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+
+#include "arc_verify.h"
+#include "arcv_internal.h"
+
+namespace arcv {
+
+constexpr uint64_t kGolden = 0x9E3779B97F4A7C15ull;
+
+__device__ __forceinline__ uint64_t fmix64(uint64_t z) {
+    z ^= z >> 30;
+    z *= 0xBF58476D1CE4E5B9ull;
+    z ^= z >> 27;
+    z *= 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+// Grid-stride over 16-byte chunks (two words) with 4 chunks in flight per
+// thread; misaligned bases assemble each word from two aligned words.
+__global__ void __launch_bounds__(256) arcv_checksum_kernel(const uint8_t *data, uint64_t bytes,
+                                                            unsigned long long *acc) {
+    const uint64_t nfull = bytes / 8;
+    const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const uint64_t nthr = (uint64_t)gridDim.x * blockDim.x;
+    const uintptr_t base = reinterpret_cast<uintptr_t>(data);
+    uint64_t s = 0, x = 0;
+    if ((base & 15) == 0) {
+        const uint4 *v = reinterpret_cast<const uint4 *>(data);
+        const uint64_t nvec = nfull / 2;
+        uint64_t c = tid;
+        for (; c + 3 * nthr < nvec; c += 4 * nthr) {
+            uint4 q[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) q[u] = __ldcs(v + c + u * nthr);
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                const uint64_t i0 = 2 * (c + u * nthr);
+                const uint64_t w0 = ((uint64_t)q[u].y << 32) | q[u].x;
+                const uint64_t w1 = ((uint64_t)q[u].w << 32) | q[u].z;
+                const uint64_t h0 = fmix64(w0 + i0 * kGolden), h1 = fmix64(w1 + (i0 + 1) * kGolden);
+                s += h0 + h1;
+                x ^= h0 ^ h1;
+            }
+        }
+        for (; c < nvec; c += nthr) {
+            const uint4 q = __ldcs(v + c);
+            const uint64_t i0 = 2 * c;
+            const uint64_t h0 = fmix64((((uint64_t)q.y << 32) | q.x) + i0 * kGolden);
+            const uint64_t h1 = fmix64((((uint64_t)q.w << 32) | q.z) + (i0 + 1) * kGolden);
+            s += h0 + h1;
+            x ^= h0 ^ h1;
+        }
+        if ((nfull & 1) && tid == 0) {  // odd last full word
+            const uint64_t i = nfull - 1;
+            const uint64_t w = reinterpret_cast<const uint64_t *>(data)[i];
+            const uint64_t h = fmix64(w + i * kGolden);
+            s += h;
+            x ^= h;
+        }
+    } else {
+        const unsigned sh = (unsigned)(base & 7) * 8;
+        const uint64_t *a = reinterpret_cast<const uint64_t *>(base & ~(uintptr_t)7);
+        for (uint64_t i = tid; i < nfull; i += nthr) {
+            uint64_t w;
+            if (sh == 0) {
+                w = a[i];
+            } else {
+                // the second word shares its 8-byte granule with byte 8i+7: mapped
+                w = (__ldcs(a + i) >> sh) | (__ldcs(a + i + 1) << (64 - sh));
+            }
+            const uint64_t h = fmix64(w + i * kGolden);
+            s += h;
+            x ^= h;
+        }
+    }
+    if ((bytes & 7) && tid == nthr - 1) {  // zero-padded tail word
+        uint64_t w = 0;
+        for (uint64_t k = 0; k < (bytes & 7); ++k) w |= (uint64_t)data[8 * nfull + k] << (8 * k);
+        const uint64_t h = fmix64(w + nfull * kGolden);
+        s += h;
+        x ^= h;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        s += __shfl_xor_sync(0xffffffffu, s, o);
+        x ^= __shfl_xor_sync(0xffffffffu, x, o);
+    }
+    if ((threadIdx.x & 31) == 0 && (s | x)) {
+        atomicAdd(acc, (unsigned long long)s);
+        atomicXor(acc + 1, (unsigned long long)x);
+    }
+}
+
+}  // namespace arcv
+
+using namespace arcv;
+
+extern "C" int arc_verify_checksum(const void *data, uint64_t bytes, uint64_t *out) {
+    if (!g_ctx) return ARC_E_NOINIT;
+    Ctx &c = *g_ctx;
+    if (!out || (bytes > 0 && (!data || classify(data, c.device) != PK_DEVICE))) {
+        set_error("checksum: device data on the library's device and a non-NULL out are required");
+        return ARC_E_INVAL;
+    }
+    unsigned long long *acc = c.counters + 5;  // 2 spare u64 counters
+    cudaError_t e = cudaMemsetAsync(acc, 0, 2 * sizeof(unsigned long long), c.stream);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(checksum)");
+    if (bytes > 0) {
+        const uint64_t chunks = (bytes + 15) / 16;
+        const uint64_t want = (chunks + 255) / 256;
+        const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(want, (uint64_t)c.num_sms * 8));
+        arcv_checksum_kernel<<<grid, 256, 0, c.stream>>>(static_cast<const uint8_t *>(data), bytes, acc);
+        e = cudaGetLastError();
+        if (e != cudaSuccess) return cuda_fail(e, "arcv_checksum_kernel launch");
+        c.launches++;
+    }
+    unsigned long long host[2];
+    e = cudaMemcpyAsync(host, acc, sizeof(host), cudaMemcpyDeviceToHost, c.stream);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpyAsync(checksum)");
+    e = cudaStreamSynchronize(c.stream);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaStreamSynchronize(checksum)");
+    out[0] = host[0];
+    out[1] = host[1];
+    return ARC_OK;
+}

@@ -337,3 +337,69 @@ def test_checks_hand_cases(oracle_mod):
     b = np.array([0, 7, -3], dtype=np.int32)
     r3 = oracle_mod.compare(a, b, "i32", 0, 0, 10, min_value=0.5)
     assert list(r3.report["index"]) == [1] and r3.max_abs_err == 2.0
+
+
+# ------------------------------------------------------- N4: checksum screen
+def _checksum_py(b: bytes):
+    """Independent pure-Python statement of the checksum definition (arbitrary ints)."""
+    M = (1 << 64) - 1
+
+    def fmix(z):
+        z ^= z >> 30
+        z = (z * 0xBF58476D1CE4E5B9) & M
+        z ^= z >> 27
+        z = (z * 0x94D049BB133111EB) & M
+        return z ^ (z >> 31)
+
+    s = x = 0
+    for i in range((len(b) + 7) // 8):
+        w = int.from_bytes(b[8 * i: 8 * i + 8].ljust(8, b"\0"), "little")
+        h = fmix((w + i * 0x9E3779B97F4A7C15) & M)
+        s = (s + h) & M
+        x ^= h
+    return s, x
+
+
+@pytest.mark.parametrize("nbytes", [0, 1, 7, 8, 9, 63, 1000, 4099])
+def test_checksum_vs_python(oracle_mod, nbytes):
+    rng = np.random.default_rng(nbytes)
+    b = rng.integers(0, 256, nbytes, dtype=np.uint8)
+    assert oracle_mod.checksum(b) == _checksum_py(b.tobytes())
+
+
+def test_checksum_properties(oracle_mod):
+    rng = np.random.default_rng(1)
+    a = rng.integers(0, 256, 1 << 16, dtype=np.uint8)
+    base = oracle_mod.checksum(a)
+    b = a.copy()
+    b[12345] ^= 1  # one bit flip changes it
+    assert oracle_mod.checksum(b) != base
+    w = a.view(np.uint64).copy()
+    w[[10, 20]] = w[[20, 10]]  # swapping two words changes it (position-dependent)
+    if w[10] != w[20]:
+        assert oracle_mod.checksum(w) != base
+    assert oracle_mod.checksum(a.copy()) == base
+
+
+def _splitmix_known():
+    rows = []
+    for line in open(os.path.join(os.path.dirname(__file__), "golden", "splitmix64_seed0.txt")):
+        line = line.split("#", 1)[0].strip()
+        if line:
+            k, v = line.split()
+            rows.append((int(k), int(v, 16)))
+    return rows
+
+
+def test_checksum_known_answer(oracle_mod):
+    """Known SplitMix64 outputs pin the finalizer, the word index term and the reductions."""
+    known = _splitmix_known()
+    words = np.full(len(known), 0x9E3779B97F4A7C15, dtype=np.uint64)
+    s, x = oracle_mod.checksum(words)
+    assert s == sum(v for _, v in known) % (1 << 64)
+    xr = 0
+    for _, v in known:
+        xr ^= v
+    assert x == xr
+    for k, v in known:  # the input generator uses the same finalizer
+        assert synth.hash64_py(0, k) == v

@@ -497,3 +497,39 @@ def test_checks_batch_and_streamed(av, orc):
     assert_same(res[1], e, "batch plain")
     g = av.compare(o.pin_memory(), r, 1e-6, 1e-5, 100, min_value=0.25, bounds=(-0.6, -0.4))
     assert_same(g, e_ck, "host streamed checked")
+
+
+# ------------------------------------------------------------- N4: checksum
+@pytest.mark.parametrize("nbytes", [0, 1, 7, 8, 15, 16, 17, 4096 * 16 + 9, (1 << 24) + 5])
+@pytest.mark.parametrize("off", [0, 1, 8, 13])
+def test_checksum_vs_oracle(av, orc, nbytes, off):
+    gen = torch.Generator().manual_seed(nbytes + off)
+    b = torch.randint(0, 256, (nbytes + off + 8,), generator=gen, dtype=torch.int32).to(torch.uint8)
+    d = b.cuda()[off:off + nbytes]
+    assert av.checksum(d) == orc.checksum(b[off:off + nbytes].numpy())
+
+
+def test_checksum_screens_c4(av, orc):
+    c4 = synth.C4(1 << 26)
+    out, ref = c4.slice(device="cuda")
+    assert av.checksum(ref) == orc.checksum(ref.cpu().numpy())
+    assert av.checksum(out) != av.checksum(ref)  # noisy output differs
+    assert av.checksum(ref.clone()) == av.checksum(ref)
+
+
+# ------------------------------------------------------ N3: selected batch
+def test_batch_selected_paper_options(av, orc):
+    regs, data = _c3_tensors()
+    items = [(o, r, reg.abs_tol, reg.rel_tol, reg.max_report, reg.name) for reg, o, r in data]
+    res = av.batch(items, options="verificationOptions=complement=0,kernels=CG:SPMUL")
+    for (reg, o, r), g in zip(data, res):
+        if reg.name in ("CG", "SPMUL"):
+            e = orc.compare(o.cpu().numpy(), r.cpu().numpy(), reg.dtype, reg.abs_tol, reg.rel_tol, reg.max_report)
+            assert_same(g, e, reg.name)
+        else:
+            assert (g.n, g.n_mismatch, g.n_reported) == (0, 0, 0)
+    res = av.batch(items, options="complement=1,kernels=JACOBI")
+    for (reg, o, r), g in zip(data, res):
+        assert (g.n == 0) == (reg.name == "JACOBI")
+    txt = av.format_result("SPMUL", "f32", 1e-6, 1e-5, res[[reg.name for reg, _, _ in data].index("SPMUL")])
+    assert txt.startswith("[arc_verify] SPMUL: FAILED")
