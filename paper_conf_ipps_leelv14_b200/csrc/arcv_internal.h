@@ -33,11 +33,18 @@ struct Ctx {
     uint64_t *active = nullptr;        size_t active_cap = 0;     // K2 active list (2 words / entry)
     uint32_t *active_cnt = nullptr;                               // [2] by parity
     uint64_t *nz_list = nullptr;                                  // K1 -> K2 pool (kPoolCap entries)
+    arc_mismatch_t *nz_ent = nullptr;                             // pool inline entries
+    uint64_t *seg_base = nullptr;      size_t seg_base_cap = 0;   // per-segment report base
+    unsigned long long lseq = 0;                                  // K1 launch numbers
+    Params deferred;                                              // K2 params of the last launch
+    bool deferred_valid = false;
     uint32_t *nz_cnt = nullptr;                                   // [2] by parity
     unsigned long long gbar_base = 0;
     uint32_t *group_cnt = nullptr;     size_t group_cap = 0;      // [2][group_cap], parity per K1
     int parity = 0;
     Acc *acc = nullptr;                size_t acc_cap = 0;
+    unsigned long long *flag_host = nullptr, *flag_dev = nullptr;  // mapped completion word
+    unsigned long long seq = 0;                                      // last finalize launch's number
     Acc *result_host = nullptr;        size_t result_host_cap = 0;   // mapped pinned
     Acc *result_dev = nullptr;                                       // its device alias
     Seg *seg_dev = nullptr;            size_t seg_dev_cap = 0;
@@ -70,7 +77,9 @@ int cuda_fail(cudaError_t e, const char *what);
 PtrKind classify(const void *p, int device);
 int validate_region(const void *out, const void *ref, uint64_t n, int dtype, double abs_tol, double rel_tol,
                     uint64_t max_report, const arc_verify_result_t *res);
-int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_t n_acc, bool finalize);
+int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_t n_acc, bool finalize,
+                    bool defer_k2);
+int wait_results(Ctx &c);
 int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_result_t *results,
               arc_mismatch_t *const *dev_reports, bool d2h_reports, Acc *summaries_out);
 
