@@ -26,7 +26,7 @@ from typing import Optional, Sequence
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libarcverify.so")
+LIB_PATH = os.environ.get("ARCV_LIB_PATH") or os.path.join(_HERE, "libarcverify.so")  # override: diagnostics
 
 ARC_OK, ARC_E_INVAL, ARC_E_NOINIT, ARC_E_CUDA, ARC_E_NCCL, ARC_E_NOMEM, ARC_E_UNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
 ARC_F32, ARC_F64, ARC_I32, ARC_I64, ARC_U8 = 0, 1, 2, 3, 4

@@ -112,9 +112,7 @@ struct SegHot {
     float at_rd, rt_rd;
     uint32_t dtype, acc_slot, cflags;
     double minv, lo, hi;
-    uint64_t index_base;
     __device__ __forceinline__ void load(const Seg &g) {
-        index_base = g.index_base;
         abs_tol = g.abs_tol; rel_tol = g.rel_tol; max_report = g.max_report;
         tile_begin = g.tile_begin; slot_begin = g.slot_begin; group_begin = g.group_begin;
         at_rd = g.at_rd; rt_rd = g.rt_rd; dtype = g.dtype; acc_slot = g.acc_slot;
@@ -486,183 +484,41 @@ __device__ __forceinline__ void flush_acc(Acc *acc_base, uint32_t slot, uint32_t
     acc.reset();
 }
 
-// Publication by the last CTA of a launch: copy the accumulators to the result
-// slots (mapped host memory), clear them for the next call, then store the
-// call's sequence number to a mapped host word that the host polls instead of
-// a stream synchronise (a system-scope fence orders the results before it).
-// Called by the consumer threads (256) of the last CTA only.
-__device__ __forceinline__ void publish_results(const Params &p, int tid) {
-    for (uint32_t k = tid; k < p.n_acc; k += kConsumerThreads) {
-        Acc a;
-        a.count = __ldcg(&p.acc[k].count);
-        a.max_abs_bits = __ldcg(&p.acc[k].max_abs_bits);
-        a.max_rel_bits = __ldcg(&p.acc[k].max_rel_bits);
-        a.pad = 0;
-        p.result[k] = a;
-        p.acc[k].count = 0;
-        p.acc[k].max_abs_bits = 0;
-        p.acc[k].max_rel_bits = 0;
+// The last CTA of the launch copies the accumulators to the result slots and
+// clears them for the next call (monotonic done counter, host-tracked base).
+// It then stores the call's sequence number to a mapped host word, which the
+// host polls instead of a stream synchronise; system-scope fences order report
+// entries written to pinned host memory (K2, `wrote_host`) and the results
+// before that word.
+__device__ __forceinline__ void finalize_launch(const Params &p, int tid, int nthreads, int *s_last,
+                                                bool wrote_host) {
+    if (tid == 0) {
+        if (wrote_host) __threadfence_system();
+        else __threadfence();
+        const unsigned long long prev = atomicAdd(p.done, 1ull);
+        *s_last = (prev - p.done_base) == (unsigned long long)(gridDim.x - 1);
     }
-    consumer_bar();
-    if (tid == 0 && p.done_flag) {
-        __threadfence_system();
-        *(volatile unsigned long long *)p.done_flag = p.seq;
-    }
-}
-
-// Exclusive scan over the 256 consumer threads (named barrier 1); returns the
-// exclusive prefix and writes the total to *total.
-__device__ __forceinline__ uint64_t cblock_excl_scan(uint64_t v, uint64_t *s_w, uint64_t *total) {
-    const int lane = threadIdx.x & 31, w = (threadIdx.x >> 5) & (kConsumerWarps - 1);
-    uint64_t inc = v;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const uint64_t y = __shfl_up_sync(0xffffffffu, inc, o);
-        if (lane >= o) inc += y;
-    }
-    if (lane == 31) s_w[w] = inc;
-    consumer_bar();
-    uint64_t base = 0, tot = 0;
-#pragma unroll
-    for (int k = 0; k < kConsumerWarps; ++k) {
-        const uint64_t x = s_w[k];
-        base += (k < w) ? x : 0ull;
-        tot += x;
-    }
-    consumer_bar();
-    *total = tot;
-    return base + inc - v;
-}
-
-// K1 tail, last CTA, launches with reporting segments (a5 for the common case).
-// 1. Each reporting segment's base report position: 0, or for a chunk of a
-//    streamed region the region's count so far minus this chunk's count.
-// 2. If the pool holds every nonzero tile (<= kPlaceMax tiles, each <= kInline
-//    mismatches, all staged inline): sort the pool by (segment, tile) with a
-//    bitonic sort in shared memory, scan the counts, and write every entry at
-//    base + prefix + rank-by-index -- the report is complete without K2.
-//    Otherwise flag the launch as pending; the host then runs K2.
-__device__ __noinline__ void k1_report_tail(const Params &p, const Seg *segs, uint8_t *scratch, int tid,
-                                            uint64_t *s_w, int *s_flag) {
-    for (uint32_t sgi = 0; sgi < p.n_segs; ++sgi) {
-        const Seg &g = segs[sgi];
-        if (g.max_report == 0) continue;
-        uint64_t base = 0;
-        if (g.flags & kSegBaseFromAcc) {
-            const uint64_t ntiles = (g.n + tile_elems(g.dtype) - 1) / tile_elems(g.dtype);
-            const uint64_t ngroups = (ntiles + kGroupTiles - 1) / kGroupTiles;
-            uint64_t t = 0;
-            for (uint64_t k = tid; k < ngroups; k += kConsumerThreads) t += __ldcg(p.group_cnt + g.group_begin + k);
-            uint64_t total;
-            cblock_excl_scan(t, s_w, &total);
-            base = __ldcg(&p.acc[g.acc_slot].count) - total;
+    if (nthreads == kConsumerThreads) consumer_bar(); else __syncthreads();
+    if (*s_last) {
+        __threadfence();
+        for (uint32_t k = tid; k < p.n_acc; k += nthreads) {
+            Acc a;
+            a.count = __ldcg(&p.acc[k].count);
+            a.max_abs_bits = __ldcg(&p.acc[k].max_abs_bits);
+            a.max_rel_bits = __ldcg(&p.acc[k].max_rel_bits);
+            a.pad = 0;
+            p.result[k] = a;
+            p.acc[k].count = 0;
+            p.acc[k].max_abs_bits = 0;
+            p.acc[k].max_rel_bits = 0;
         }
-        if (tid == 0) p.seg_base[sgi] = base;
-    }
-    const uint32_t n = *(volatile uint32_t *)p.nz_cnt;
-    if (tid == 0) *s_flag = (n <= (uint32_t)kPlaceMax && p.n_segs < 4096u && !(p.flags & kFlagNoK1Place)) ? 1 : 0;
-    consumer_bar();
-    uint64_t *v = reinterpret_cast<uint64_t *>(scratch);       // sort keys
-    uint64_t *ex = v + kPlaceMax;                               // exclusive prefix, sorted order
-    uint32_t N = 2;
-    while (N < n) N <<= 1;
-    if (*s_flag) {
-        for (uint32_t i = tid; i < N; i += kConsumerThreads) {
-            uint64_t key = ~0ull;
-            if (i < n) {
-                const uint64_t k0 = __ldcg(p.nz_list + 2 * i), c = __ldcg(p.nz_list + 2 * i + 1);
-                if (c > (uint64_t)kInline) *s_flag = 0;  // a dense tile: entries were not staged
-                key = ((k0 >> 40) << 52) | ((k0 & ((1ull << 40) - 1)) << 11) | i;
+        if (p.done_flag) {
+            if (nthreads == kConsumerThreads) consumer_bar(); else __syncthreads();
+            if (tid == 0) {
+                __threadfence_system();
+                *(volatile unsigned long long *)p.done_flag = p.seq;
             }
-            v[i] = key;
         }
-    }
-    consumer_bar();
-    if (!*s_flag) {
-        if (tid == 0) *p.pending_host = p.lseq;  // the host runs K2
-        return;
-    }
-    for (uint32_t k = 2; k <= N; k <<= 1) {
-        for (uint32_t j = k >> 1; j > 0; j >>= 1) {
-            for (uint32_t i = tid; i < N; i += kConsumerThreads) {
-                const uint32_t ixj = i ^ j;
-                if (ixj > i) {
-                    const uint64_t a = v[i], b = v[ixj];
-                    if ((a > b) == ((i & k) == 0)) {
-                        v[i] = b;
-                        v[ixj] = a;
-                    }
-                }
-            }
-            consumer_bar();
-        }
-    }
-    // exclusive scan of counts in sorted order: 4 consecutive keys per thread
-    uint64_t c4[4], local = 0;
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-        const uint32_t j = tid * 4 + q;
-        c4[q] = j < n ? __ldcg(p.nz_list + 2 * (v[j] & 2047) + 1) : 0;
-        local += c4[q];
-    }
-    uint64_t total;
-    uint64_t run = cblock_excl_scan(local, s_w, &total);
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-        const uint32_t j = tid * 4 + q;
-        if (j < n) ex[j] = run;
-        run += c4[q];
-    }
-    consumer_bar();
-    for (uint32_t j = tid; j < n; j += kConsumerThreads) {
-        const uint64_t key = v[j];
-        const uint32_t idx = (uint32_t)(key & 2047), sgi = (uint32_t)(key >> 52);
-        const uint64_t lt = (key >> 11) & ((1ull << 41) - 1);
-        uint32_t lo = 0, hi = j;  // first sorted position of this segment
-        while (lo < hi) {
-            const uint32_t mid = (lo + hi) >> 1;
-            if ((v[mid] >> 52) < sgi) lo = mid + 1; else hi = mid;
-        }
-        const Seg &g = segs[sgi];
-        const uint64_t pos0 = p.seg_base[sgi] + ex[j] - ex[lo];
-        const uint32_t c = (uint32_t)__ldcg(p.nz_list + 2 * idx + 1);
-        p.tile_cnt[g.slot_begin + lt] = 0u;  // clean for the next call
-        if (pos0 >= g.max_report) continue;
-        arc_mismatch_t e[kInline];
-        for (uint32_t r = 0; r < c; ++r) {  // insertion sort by index (c <= kInline)
-            arc_mismatch_t x = p.nz_ent[(size_t)idx * kInline + r];
-            uint32_t q = r;
-            while (q > 0 && e[q - 1].index > x.index) {
-                e[q] = e[q - 1];
-                --q;
-            }
-            e[q] = x;
-        }
-        for (uint32_t r = 0; r < c && pos0 + r < g.max_report; ++r) g.report[pos0 + r] = e[r];
-    }
-    __threadfence_system();  // entries may live in pinned host memory
-    consumer_bar();
-    if (tid == 0) *p.resolved = p.lseq;
-}
-
-// Write this thread's mismatch entries of a tile (bits in `mask`, same layout as
-// eval_tile) to consecutive slots at `dst`, reading the values from the stage.
-__device__ __noinline__ void stage_entries(const uint8_t *so, const uint8_t *sr, const StageInfo &si,
-                                           const SegHot &g, int ctid, uint64_t mask, arc_mismatch_t *dst) {
-    const uint32_t es = elem_size(g.dtype);
-    const int epv = (int)(16u / es);
-    uint64_t m = mask;
-    while (m) {
-        const int b = __ffsll((long long)m) - 1;
-        m &= m - 1;
-        const uint32_t te = (uint32_t)(((b / epv) * kConsumerThreads + ctid) * epv + (b % epv));
-        uint64_t ob = 0, rb = 0;
-        memcpy(&ob, so + si.off_o + te * es, es);  // little-endian: zero-extended raw bits
-        memcpy(&rb, sr + si.off_r + te * es, es);
-        dst->index = g.index_base + si.elem_begin + te;
-        dst->out_bits = ob;
-        dst->ref_bits = rb;
-        ++dst;
     }
 }
 
@@ -675,11 +531,8 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
     __shared__ StageInfo info[S];
     __shared__ uint64_t s_red_u[kConsumerWarps][2];
     __shared__ double s_red_d[kConsumerWarps][2];
-    __shared__ int s_last, s_flag;
-    __shared__ uint64_t s_scan_w[kConsumerWarps];
+    __shared__ int s_last;
     __shared__ uint32_t s_tile[S];
-    __shared__ uint32_t s_ecnt[S];
-    __shared__ arc_mismatch_t s_ent[S][kInline];
 
     const Seg *segs = p.segs ? p.segs : p.inline_segs;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -687,7 +540,6 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) {
             s_tile[s] = 0u;
-            s_ecnt[s] = 0u;
             mbar_init(&full_bar[s], 1);
             mbar_init(&empty_bar[s], kConsumerWarps);
         }
@@ -758,56 +610,30 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
         const uint32_t cnt = (uint32_t)__popcll(mask);
         acc.count += cnt;
         if (g.max_report != 0) {
-            // Per-tile bookkeeping for the ordered report (a5):
-            //  * a sparse tile's mismatch entries (<= kInline) are staged in shared
-            //    memory now, while the stage still holds the values;
-            //  * warps fold their counts into the stage's word (arrivals << 24 |
-            //    count); the last warp publishes the tile: tile/group counts (K2's
-            //    dense path) and, for the pool, {tile, count} + the inline entries.
+            // Per-tile count for K2: warps fold their counts into the stage's
+            // shared word (arrivals << 24 | count); the last warp publishes the
+            // tile (2 global atomics per tile with mismatches, none otherwise)
+            // and clears the word before the stage can be reused.
             const uint32_t wc = __reduce_add_sync(0xffffffffu, cnt);
-            if (wc != 0) {
-                uint32_t pos = 0;
-                if (lane == 0) pos = atomicAdd(&s_ecnt[s], wc);
-                pos = __shfl_sync(0xffffffffu, pos, 0);
-                if (pos + wc <= (uint32_t)kInline) {
-                    uint32_t incl = cnt;
-#pragma unroll
-                    for (int o = 1; o < 32; o <<= 1) {
-                        const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
-                        if (lane >= o) incl += y;
-                    }
-                    stage_entries(so, so + kStageArrayBytes, si, g, ctid, mask, &s_ent[s][pos + incl - cnt]);
-                }
-                __threadfence_block();
-            }
-            uint32_t old = 0;
-            if (lane == 0) old = atomicAdd(&s_tile[s], (1u << 24) | wc);
-            old = __shfl_sync(0xffffffffu, old, 0);
-            if ((old >> 24) == kConsumerWarps - 1) {  // warp-uniform: this warp publishes the tile
-                __threadfence_block();
-                const uint32_t tc = (old & 0xffffffu) + wc;
-                uint32_t k = ~0u;
-                if (tc != 0 && lane == 0) {
-                    const uint64_t lt = si.tile - g.tile_begin;
-                    atomicAdd(p.tile_cnt + g.slot_begin + lt, tc);
-                    atomicAdd(p.group_cnt + g.group_begin + lt / kGroupTiles, tc);
-                    // pool of nonzero tiles (checked before the atomic so a dense
-                    // call stops touching it)
-                    if (*(volatile uint32_t *)p.nz_cnt < (uint32_t)kPoolCap) {
-                        k = atomicAdd(p.nz_cnt, 1u);
-                        if (k < (uint32_t)kPoolCap) {
-                            p.nz_list[2 * k] = ((uint64_t)si.seg << 40) | lt;
-                            p.nz_list[2 * k + 1] = tc;
+            if (lane == 0) {
+                const uint32_t old = atomicAdd(&s_tile[s], (1u << 24) | wc);
+                if ((old >> 24) == kConsumerWarps - 1) {
+                    const uint32_t tc = (old & 0xffffffu) + wc;
+                    s_tile[s] = 0u;
+                    if (tc != 0) {
+                        const uint64_t lt = si.tile - g.tile_begin;
+                        atomicAdd(p.tile_cnt + g.slot_begin + lt, tc);
+                        atomicAdd(p.group_cnt + g.group_begin + lt / kGroupTiles, tc);
+                        // short list of nonzero tiles for K2's pool path (checked
+                        // before the atomic so a dense call stops touching it)
+                        if (*(volatile uint32_t *)p.nz_cnt < (uint32_t)kPoolCap) {
+                            const uint32_t k = atomicAdd(p.nz_cnt, 1u);
+                            if (k < (uint32_t)kPoolCap) {
+                                p.nz_list[2 * k] = ((uint64_t)si.seg << 40) | lt;
+                                p.nz_list[2 * k + 1] = tc;
+                            }
                         }
                     }
-                }
-                k = __shfl_sync(0xffffffffu, k, 0);
-                if (k < (uint32_t)kPoolCap && tc <= (uint32_t)kInline && (uint32_t)lane < tc)
-                    p.nz_ent[(size_t)k * kInline + lane] = s_ent[s][lane];
-                __syncwarp();
-                if (lane == 0) {
-                    s_tile[s] = 0u;
-                    s_ecnt[s] = 0u;
                 }
             }
         }
@@ -816,17 +642,7 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
         if (lane == 0) mbar_arrive(&empty_bar[s]);  // stage may be refilled now
     }
     if (cur >= 0) flush_acc(p.acc, g.acc_slot, g.dtype, acc, ctid, s_red_u, s_red_d);
-    // the last CTA to finish (monotonic done counter, host-tracked base)
-    if (ctid == 0) {
-        __threadfence();
-        const unsigned long long prev = atomicAdd(p.done, 1ull);
-        s_last = (prev - p.done_base) == (unsigned long long)(gridDim.x - 1);
-    }
-    consumer_bar();
-    if (!s_last) return;
-    __threadfence();
-    if (p.has_report) k1_report_tail(p, segs, smem, ctid, s_scan_w, &s_flag);
-    if (p.finalize) publish_results(p, ctid);
+    if (p.finalize) finalize_launch(p, ctid, kConsumerThreads, &s_last, false);
 }
 
 // --------------------------------------------------------------- K2 helpers
@@ -988,6 +804,7 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
     __shared__ uint64_t s_loc_key[kPoolLocal];
     __shared__ uint64_t s_loc_pre[kPoolLocal];
     __shared__ uint32_t s_n;
+    __shared__ int s_last;
     uint64_t *s_pkey = reinterpret_cast<uint64_t *>(smem + 2 * kStageBytes);
     uint32_t *s_pcnt = reinterpret_cast<uint32_t *>(s_pkey + kPoolCap);
 
@@ -1039,10 +856,6 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
         }
     };
 
-    if (*(volatile unsigned long long *)p.resolved == p.lseq) {  // K1 placed the report itself
-        if (tid == 0) atomicAdd(p.gbar, 1ull);  // keep the barrier bookkeeping
-        return;
-    }
     const uint32_t n_nz = *(volatile uint32_t *)p.nz_cnt;
     if (n_nz <= (uint32_t)kPoolCap) {
         // ------------------------------------------------------ pool path
@@ -1058,15 +871,20 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
         for (uint32_t k = blockIdx.x; k < n_nz; k += gridDim.x) {
             const uint64_t key = s_pkey[k];
             const uint64_t seg = key >> 40, lt = key & kLtMask;
-            uint64_t pre = 0;
+            uint64_t pre = 0, segtot = 0;
             for (uint32_t i = tid; i < n_nz; i += kConsumerThreads) {
                 const uint64_t ki = s_pkey[i];
-                if ((ki >> 40) == seg && (ki & kLtMask) < lt) pre += s_pcnt[i];
+                if ((ki >> 40) == seg) {
+                    segtot += s_pcnt[i];
+                    pre += ((ki & kLtMask) < lt) ? s_pcnt[i] : 0u;
+                }
             }
-            uint64_t pre_tot;
+            uint64_t pre_tot, seg_tot;
             block_excl_scan(pre, s_w, &pre_tot);
+            block_excl_scan(segtot, s_w, &seg_tot);
             const Seg &g = segs[seg];
-            const uint64_t base = __ldcg(p.seg_base + seg);
+            uint64_t base = 0;
+            if (g.flags & kSegBaseFromAcc) base = __ldcg(&p.acc[g.acc_slot].count) - seg_tot;
             if (tid == 0) {
                 p.tile_cnt[g.slot_begin + lt] = 0u;  // clean for the next call
                 if (base + pre_tot < g.max_report && s_n < (uint32_t)kPoolLocal) {
@@ -1092,7 +910,8 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
             uint64_t total;
             block_excl_scan(tot, s_w, &total);
             if (total == 0) continue;  // uniform: nothing to report or to clear
-            const uint64_t base = __ldcg(p.seg_base + sgi);
+            uint64_t base = 0;
+            if (g.flags & kSegBaseFromAcc) base = __ldcg(&p.acc[g.acc_slot].count) - total;
 
             uint64_t run = base, ord_run = 0;
             for (uint64_t c0 = 0; c0 < ngroups; c0 += kGroupTiles) {
@@ -1141,7 +960,7 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
         process(mine, [&](uint32_t j) { return __ldcg(p.active + 2 * (blockIdx.x + j * gridDim.x)); },
                 [&](uint32_t j) { return __ldcg(p.active + 2 * (blockIdx.x + j * gridDim.x) + 1); });
     }
-    __threadfence_system();  // report entries may live in pinned host memory
+    if (p.finalize) finalize_launch(p, tid, kConsumerThreads, &s_last, p.report_host != 0);
 }
 
 }  // namespace arcv

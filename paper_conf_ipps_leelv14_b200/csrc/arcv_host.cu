@@ -207,27 +207,10 @@ static Seg make_seg(const void *out, const void *ref, uint64_t n, uint32_t dtype
 }
 
 // ------------------------------------------------------------------ launch
-static int launch_compact(Ctx &c, const Params &p) {
-    const uint32_t grid2 = (uint32_t)c.num_sms;
-    Params q = p;
-    q.gbar_base = c.gbar_base;
-    void *args[] = {&q};
-    cudaError_t e = cudaLaunchCooperativeKernel((const void *)arcv_compact_kernel, dim3(grid2),
-                                                dim3(kConsumerThreads), args, kCompactSmem, c.stream);
-    if (e != cudaSuccess) return cuda_fail(e, "arcv_compact_kernel cooperative launch");
-    c.launches++;
-    c.gbar_base += grid2;
-    return ARC_OK;
-}
-
-// One K1 over `segs` (fills each seg's tile_begin / group_begin).  Its last CTA
-// places the report itself in the common sparse case; otherwise K2 must run:
-// immediately after K1 when `defer_k2` is false (streamed chunks: K2 returns
-// at once if K1 resolved), or -- for a device-resident call -- only if the
-// host finds the launch pending after the results are in (run_local).
-// Accumulator slots [acc_lo, acc_lo + n_acc) are published when `finalize`.
-int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_t n_acc, bool finalize,
-                    bool defer_k2) {
+// One K1 (+ K2 when any segment wants a report) over `segs`.  Fills each seg's
+// tile_begin / group_begin.  Accumulator slots [acc_lo, acc_lo + n_acc) are
+// published to the result slots when `finalize`.
+int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_t n_acc, bool finalize) {
     uint64_t tiles = 0, groups = 0;
     bool need_compact = false;
     for (uint32_t k = 0; k < n_segs; ++k) {
@@ -247,8 +230,7 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
         if (st) return st;
         c.group_cap = cap2 / 2;
     }
-    int st = grow_device(&c.seg_base, &c.seg_base_cap, std::max<uint32_t>(n_segs, 64), false, c.stream);
-    if (st) return st;
+    int st = ARC_OK;
     Params p;
     memset(&p, 0, sizeof(p));
     if (n_segs <= (uint32_t)kMaxInlineSegs) {
@@ -279,22 +261,18 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
     p.active_cnt = c.active_cnt + c.parity;
     p.active_cnt_zero = c.active_cnt + (c.parity ^ 1);
     p.nz_list = c.nz_list;
-    p.nz_ent = c.nz_ent;
     p.nz_cnt = c.nz_cnt + c.parity;
     p.nz_cnt_zero = c.nz_cnt + (c.parity ^ 1);
-    p.seg_base = c.seg_base;
-    p.resolved = c.counters + 7;
-    p.pending_host = c.flag_dev + 1;
-    p.lseq = ++c.lseq;
     p.gbar = c.counters + 2;
     p.gbar_base = c.gbar_base;
     p.acc = c.acc + acc_lo;
     p.result = c.result_dev + acc_lo;
-    p.finalize = finalize ? 1 : 0;
-    p.has_report = need_compact ? 1u : 0u;
+    p.finalize = (finalize && !need_compact) ? 1 : 0;
     p.flags = (uint32_t)c.flags;
-    p.done_flag = c.flag_dev;
+    p.done_flag = (c.flags & 8) ? nullptr : c.flag_dev;  // ARCV_FLAGS bit 3 (diagnostic): stream sync
     if (finalize) p.seq = ++c.seq;  // the host waits for the last finalize launch's number
+    for (uint32_t k = 0; k < n_segs; ++k)
+        if (segs[k].report && classify(segs[k].report, c.device) != PK_DEVICE) p.report_host = 1;
 
     const uint64_t max_grid = (uint64_t)c.num_sms * (uint64_t)c.ctas_per_sm;
     const uint32_t grid = (uint32_t)std::min<uint64_t>(tiles, max_grid);
@@ -306,16 +284,18 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
     if (e != cudaSuccess) return cuda_fail(e, "arcv_stream_kernel launch");
     c.launches++;
     c.ticket_base += tiles + grid;
-    c.done_base += grid;  // every K1 launch elects a last CTA
-    c.deferred_valid = false;
+    if (p.finalize) c.done_base += grid;
     if (need_compact) {
-        if (defer_k2) {
-            c.deferred = p;
-            c.deferred_valid = true;
-        } else {
-            st = launch_compact(c, p);
-            if (st) return st;
-        }
+        p.finalize = finalize ? 1 : 0;
+        p.done_base = c.done_base;
+        const uint32_t grid2 = (uint32_t)c.num_sms;
+        void *args[] = {&p};
+        e = cudaLaunchCooperativeKernel((const void *)arcv_compact_kernel, dim3(grid2), dim3(kConsumerThreads), args,
+                                        kCompactSmem, c.stream);
+        if (e != cudaSuccess) return cuda_fail(e, "arcv_compact_kernel cooperative launch");
+        c.launches++;
+        c.gbar_base += grid2;
+        if (finalize) c.done_base += grid2;
     }
     if (timed) {
         CK(cudaEventRecord(c.ev[c.n_ev][1], c.stream));
@@ -325,24 +305,14 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
     return ARC_OK;
 }
 
-// After a deferred launch's results are in: run K2 if its K1 could not place
-// the report (dense or overflowing pool), and wait for it.
-static int finish_deferred(Ctx &c) {
-    if (!c.deferred_valid) return ARC_OK;
-    c.deferred_valid = false;
-    if (__atomic_load_n(c.flag_host + 1, __ATOMIC_ACQUIRE) != c.deferred.lseq) return ARC_OK;
-    int st = launch_compact(c, c.deferred);
-    if (st) return st;
-    // fold K2 into the call's timing window: move the last window's end event
-    if (c.timing && c.n_ev > 0) CK(cudaEventRecord(c.ev[c.n_ev - 1][1], c.stream));
-    CK(cudaStreamSynchronize(c.stream));
-    return ARC_OK;
-}
-
 // Wait until the last finalize launch has published its results: poll the
 // mapped completion word (cheaper to wake on than a stream synchronise), and
 // fall back to the stream's status so errors surface and nothing can hang.
 int wait_results(Ctx &c) {
+    if (c.flags & 8) {
+        CK(cudaStreamSynchronize(c.stream));
+        return ARC_OK;
+    }
     const unsigned long long want = c.seq;
     for (uint64_t it = 1;; ++it) {
         if (__atomic_load_n(c.flag_host, __ATOMIC_ACQUIRE) == want) return ARC_OK;
@@ -438,7 +408,7 @@ static int stream_region(Ctx &c, const arc_verify_region_t &r, bool out_dev, boo
         CK(cudaStreamWaitEvent(c.stream, c.ev_copy[b], 0));
         Seg g = make_seg(po, pr, ne, dtype, r.abs_tol, r.rel_tol, r.max_report, report, slot_base + e0 / te, e0, 0,
                          kSegBaseFromAcc, r.check);
-        int st = launch_segments(c, &g, 1, acc_slot, 1, ci + 1 == nchunks, false);
+        int st = launch_segments(c, &g, 1, acc_slot, 1, ci + 1 == nchunks);
         if (st) return st;
         CK(cudaEventRecord(c.ev_free[b], c.stream));
     }
@@ -524,10 +494,8 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
     for (size_t k = 0; k < R; ++k)
         if (plan[k].stream && regs[k].n > 0) slot_of[k] = next_slot++;
 
-    bool any_streamed = false;
-    for (size_t k = 0; k < R; ++k) any_streamed |= plan[k].stream && regs[k].n > 0;
     if (!segs.empty()) {  // one grid over every device-resident region (a7)
-        st = launch_segments(c, segs.data(), (uint32_t)segs.size(), 0, n_dev_slots, true, !any_streamed);
+        st = launch_segments(c, segs.data(), (uint32_t)segs.size(), 0, n_dev_slots, true);
         if (st) return st;
     }
     for (size_t k = 0; k < R; ++k) {
@@ -538,14 +506,8 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
     }
     const uint32_t n_slots = next_slot;
     if (n_slots) {  // result slots are mapped host memory
-        if (any_streamed) {
-            CK(cudaStreamSynchronize(c.stream));  // the last chunk's K2 follows its K1
-        } else {
-            st = wait_results(c);
-            if (st) return st;
-            st = finish_deferred(c);
-            if (st) return st;
-        }
+        st = wait_results(c);
+        if (st) return st;
     }
     if (c.timing) {
         st = collect_timing(c);
@@ -663,6 +625,12 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
     if (occ < 1) { set_error("kernel does not fit on an SM (smem %zu)", smem); return ARC_E_UNSUPPORTED; }
     const int cap = env_int("ARCV_CTAS_PER_SM", 0);
     c->ctas_per_sm = cap > 0 ? std::min(cap, occ) : occ;
+    if (env_int("ARCV_VERBOSE", 0)) {
+        cudaFuncAttributes fa;
+        CK(cudaFuncGetAttributes(&fa, kf));
+        fprintf(stderr, "[arcv] sms=%d stages=%d ctas/sm=%d (occupancy %d) regs=%d static_smem=%zu dyn_smem=%zu local=%zu\n",
+                c->num_sms, c->stages, c->ctas_per_sm, occ, fa.numRegs, fa.sharedSizeBytes, smem, fa.localSizeBytes);
+    }
     // counters: [0] tile tickets, [1] finished CTAs, [2] K2 grid barrier,
     // [3] 2 x u32 active-list lengths, [4] 2 x u32 pool lengths (by parity)
     e = cudaMalloc(&c->counters, 8 * sizeof(unsigned long long));
@@ -671,14 +639,11 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
     e = cudaHostAlloc(reinterpret_cast<void **>(&c->flag_host), 64, cudaHostAllocMapped);
     if (e != cudaSuccess) { cudaGetLastError(); set_error("cudaHostAlloc(flag)"); return ARC_E_NOMEM; }
     c->flag_host[0] = 0;
-    c->flag_host[1] = 0;
     CK(cudaHostGetDevicePointer(reinterpret_cast<void **>(&c->flag_dev), c->flag_host, 0));
     c->active_cnt = reinterpret_cast<uint32_t *>(c->counters + 3);
     c->nz_cnt = reinterpret_cast<uint32_t *>(c->counters + 4);
     e = cudaMalloc(&c->nz_list, 2 * kPoolCap * sizeof(uint64_t));
     if (e != cudaSuccess) { cudaGetLastError(); set_error("cudaMalloc pool list"); return ARC_E_NOMEM; }
-    e = cudaMalloc(&c->nz_ent, (size_t)kPoolCap * kInline * sizeof(arc_mismatch_t));
-    if (e != cudaSuccess) { cudaGetLastError(); set_error("cudaMalloc pool entries"); return ARC_E_NOMEM; }
     CK(cudaStreamSynchronize(c->stream));
     g_ctx = c;
     c->sharded = o.nccl_unique_id != nullptr;
@@ -701,8 +666,6 @@ int arc_verify_finalize(void) {
     cudaFree(c->tile_cnt);
     cudaFree(c->active);
     cudaFree(c->nz_list);
-    cudaFree(c->nz_ent);
-    cudaFree(c->seg_base);
     cudaFree(c->group_cnt);
     cudaFree(c->acc);
     cudaFree(c->seg_dev);
@@ -811,9 +774,9 @@ int arc_verify_probe_read(const void *a, const void *b, uint64_t bytes, int iter
     CK(cudaEventCreate(&e0));
     CK(cudaEventCreate(&e1));
     Seg g = make_seg(a, b, bytes, ARC_U8, 0.0, 0.0, 0, nullptr, 0, 0, 0, 0);
-    st = launch_segments(c, &g, 1, 0, 1, true, false);  // warm-up
+    st = launch_segments(c, &g, 1, 0, 1, true);  // warm-up
     CK(cudaEventRecord(e0, c.stream));
-    for (int i = 0; i < iters && !st; ++i) st = launch_segments(c, &g, 1, 0, 1, true, false);
+    for (int i = 0; i < iters && !st; ++i) st = launch_segments(c, &g, 1, 0, 1, true);
     CK(cudaEventRecord(e1, c.stream));
     CK(cudaEventSynchronize(e1));
     float ms = 0.f;

@@ -33,11 +33,6 @@ struct Ctx {
     uint64_t *active = nullptr;        size_t active_cap = 0;     // K2 active list (2 words / entry)
     uint32_t *active_cnt = nullptr;                               // [2] by parity
     uint64_t *nz_list = nullptr;                                  // K1 -> K2 pool (kPoolCap entries)
-    arc_mismatch_t *nz_ent = nullptr;                             // pool inline entries
-    uint64_t *seg_base = nullptr;      size_t seg_base_cap = 0;   // per-segment report base
-    unsigned long long lseq = 0;                                  // K1 launch numbers
-    Params deferred;                                              // K2 params of the last launch
-    bool deferred_valid = false;
     uint32_t *nz_cnt = nullptr;                                   // [2] by parity
     unsigned long long gbar_base = 0;
     uint32_t *group_cnt = nullptr;     size_t group_cap = 0;      // [2][group_cap], parity per K1
@@ -77,8 +72,7 @@ int cuda_fail(cudaError_t e, const char *what);
 PtrKind classify(const void *p, int device);
 int validate_region(const void *out, const void *ref, uint64_t n, int dtype, double abs_tol, double rel_tol,
                     uint64_t max_report, const arc_verify_result_t *res);
-int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_t n_acc, bool finalize,
-                    bool defer_k2);
+int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_t n_acc, bool finalize);
 int wait_results(Ctx &c);
 int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_result_t *results,
               arc_mismatch_t *const *dev_reports, bool d2h_reports, Acc *summaries_out);

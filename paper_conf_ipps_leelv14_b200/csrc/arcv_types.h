@@ -18,13 +18,10 @@ constexpr int kMaxInlineSegs = 8;
 constexpr int kGroupTiles = 256;                    // tiles per group counter
 constexpr int kPoolCap = 2048;                      // K2 pool path: max listed nonzero tiles
 constexpr int kPoolLocal = 64;                      // per-CTA share of the pool (grid >= 32)
-constexpr int kInline = 8;                          // mismatch entries kept inline per pool tile
-constexpr int kPlaceMax = 1024;                     // K1 places the pool itself up to this many tiles
 static_assert(kVecPerThread == 4, "packed-scan layout assumes 4 vectors per thread");
 static_assert(kGroupTiles == kConsumerThreads, "K2 scans one group per block pass");
 
-constexpr uint32_t kFlagProbe = 2u;
-constexpr uint32_t kFlagNoK1Place = 4u;  // Params.flags (diagnostic, ARCV_FLAGS=4): always defer placement to K2       // Params.flags: stream only, no predicate (read probe)
+constexpr uint32_t kFlagProbe = 2u;       // Params.flags: stream only, no predicate (read probe)
 constexpr uint32_t kSegBaseFromAcc = 1u;  // chunk of a streamed region: prefix base = acc count - own total
 
 // One contiguous piece of one region (a whole region, or one chunk of a region
@@ -72,11 +69,6 @@ struct Params {
     uint32_t *active_cnt;     // this launch's list length
     uint32_t *active_cnt_zero;  // the other parity, zeroed by K1 for the next launch
     uint64_t *nz_list;        // K1 -> K2 pool: {seg << 40 | tile, count} of nonzero tiles
-    arc_mismatch_t *nz_ent;   // pool: up to kInline entries per listed tile (unordered)
-    uint64_t *seg_base;       // per segment: report position of its first mismatch (K1 tail -> K2)
-    unsigned long long *resolved;      // device word: = lseq when K1 placed the report itself
-    unsigned long long *pending_host;  // mapped host word: = lseq when K2 must run
-    unsigned long long lseq;           // this launch's number
     uint32_t *nz_cnt;         // this launch's pool length (may exceed kPoolCap: overflow)
     uint32_t *nz_cnt_zero;    // the other parity
     unsigned long long *gbar; // K2 grid barrier counter (monotonic)
@@ -85,9 +77,9 @@ struct Params {
     Acc *result;
     unsigned long long *done_flag;  // mapped host word: seq is stored when the call's results are final
     unsigned long long seq;
+    uint32_t report_host;           // some report lives in pinned host memory (system-scope fences)
     int finalize;
     uint32_t flags;
-    uint32_t has_report;      // some segment has max_report > 0
     Seg inline_segs[kMaxInlineSegs];
 };
 

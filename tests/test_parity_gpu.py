@@ -237,12 +237,14 @@ def test_host_inputs_streamed(av, orc, where):
 
 
 # ------------------------------------------------------------ stage variants
-@pytest.mark.parametrize("stages,ctas", [(2, 0), (4, 0), (6, 0), (3, 1)])
-def test_launch_geometry_invariance(orc, stages, ctas):
+@pytest.mark.parametrize("stages,ctas,flags", [(2, 0, 0), (4, 0, 0), (6, 0, 0), (3, 1, 0), (3, 0, 8)])
+def test_launch_geometry_invariance(orc, stages, ctas, flags):
+    """Stage counts, CTAs per SM, and (flags=8) stream-sync instead of the completion word."""
     import paper_conf_ipps_leelv14_b200 as av
 
     av.finalize()
     os.environ["ARCV_STAGES"], os.environ["ARCV_CTAS_PER_SM"] = str(stages), str(ctas)
+    os.environ["ARCV_FLAGS"] = str(flags)
     try:
         av.init(0)
         c1 = synth.C1()
@@ -250,9 +252,13 @@ def test_launch_geometry_invariance(orc, stages, ctas):
         run_both(av, orc, out.cuda(), ref.cuda(), "f32", 1e-6, 1e-5, 30, f"stages={stages}")
         o5, r5 = synth.C5(1 << 22).slice(device="cuda")
         run_both(av, orc, o5, r5, "i32", 0, 0, 5000, f"c5 stages={stages}")
+        c4 = synth.C4(1 << 22)
+        o4, r4 = c4.slice(device="cuda")
+        run_both(av, orc, o4, r4, "f64", 1e-6, 1e-5, 300, f"c4 stages={stages} flags={flags}")
+        run_both(av, orc, o4.cpu().pin_memory(), r4, "f64", 1e-6, 1e-5, 300, f"c4 host flags={flags}")
     finally:
         av.finalize()
-        del os.environ["ARCV_STAGES"], os.environ["ARCV_CTAS_PER_SM"]
+        del os.environ["ARCV_STAGES"], os.environ["ARCV_CTAS_PER_SM"], os.environ["ARCV_FLAGS"]
         av.init(0)
 
 
