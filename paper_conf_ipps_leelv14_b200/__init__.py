@@ -396,6 +396,69 @@ def compare(out, ref, abs_tol: float = 0.0, rel_tol: float = 0.0, max_report: in
     return Result(res.n, res.n_mismatch, res.max_abs_err, res.max_rel_err, nr, rep)
 
 
+class Prepared:
+    """A comparison whose arguments are validated and marshalled once.
+
+    ``p = prepare(out, ref, abs_tol, rel_tol, max_report, report=...)`` then each
+    ``p()`` is one arc_verify_compare(_ex) call through pre-built ctypes
+    arguments -- for callers that verify the same buffers repeatedly (an
+    iterative solver checked every step; a benchmark loop).  The tensors and the
+    report buffer must stay alive and in place.
+    """
+
+    __slots__ = ("_fn", "_args", "_res", "_rep", "_keep")
+
+    def __init__(self, out, ref, abs_tol=0.0, rel_tol=0.0, max_report=1 << 20, report=None, n=None,
+                 min_value=None, bounds=None):
+        if _TORCH_CODES is None:
+            dtype_code(out)
+        code = _TORCH_CODES.get(out.dtype)
+        if code is None or out.dtype != ref.dtype:
+            raise TypeError(f"unsupported or mismatched dtypes {out.dtype} / {ref.dtype}")
+        if n is None:
+            n = out.numel()
+            if ref.numel() != n:
+                raise ValueError("size mismatch")
+        if n and not (out.is_contiguous() and ref.is_contiguous()):
+            raise ValueError("tensors must be contiguous")
+        if report is None:
+            report, ptr = _report_buffer(min(int(max_report), n))
+        elif isinstance(report, np.ndarray):
+            ptr = report.ctypes.data
+        else:
+            ptr = report.data_ptr()
+        self._rep = report
+        self._res = arc_verify_result_t()
+        self._res.report = ptr if max_report > 0 else None
+        ck = make_check(min_value, bounds)
+        args = [ctypes.c_void_p(out.data_ptr() if n else None), ctypes.c_void_p(ref.data_ptr() if n else None),
+                ctypes.c_uint64(n), ctypes.c_int(code), ctypes.c_double(abs_tol), ctypes.c_double(rel_tol),
+                ctypes.c_uint64(max_report)]
+        if ck is None:
+            self._fn = _lib.arc_verify_compare
+        else:
+            self._fn = _lib.arc_verify_compare_ex
+            args.append(ctypes.byref(ck))
+        args.append(ctypes.byref(self._res))
+        self._args = tuple(args)
+        self._keep = (out, ref, ck)
+
+    def __call__(self) -> Result:
+        st = self._fn(*self._args)
+        if st:
+            raise ArcVerifyError(st, "arc_verify_compare")
+        r = self._res
+        nr = r.n_reported
+        rep = self._rep[:nr] if isinstance(self._rep, np.ndarray) else self._rep
+        return Result(r.n, r.n_mismatch, r.max_abs_err, r.max_rel_err, nr, rep)
+
+
+def prepare(out, ref, abs_tol: float = 0.0, rel_tol: float = 0.0, max_report: int = 1 << 20, report=None,
+            n: Optional[int] = None, min_value: Optional[float] = None, bounds=None) -> Prepared:
+    """Validate and marshal a comparison once; call the result to run it (see Prepared)."""
+    return Prepared(out, ref, abs_tol, rel_tol, max_report, report, n, min_value, bounds)
+
+
 def batch(regions, options: Optional[str] = None, select: bool = False) -> list[Result]:
     """regions: iterable of (out, ref, abs_tol, rel_tol, max_report[, name[, check]]) with torch
     tensors; ``check`` is an arc_verify_check_t (see make_check) or None."""

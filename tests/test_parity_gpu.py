@@ -539,3 +539,30 @@ def test_batch_selected_paper_options(av, orc):
         assert (g.n == 0) == (reg.name == "JACOBI")
     txt = av.format_result("SPMUL", "f32", 1e-6, 1e-5, res[[reg.name for reg, _, _ in data].index("SPMUL")])
     assert txt.startswith("[arc_verify] SPMUL: FAILED")
+
+
+def test_prepared_call(av, orc):
+    c1 = synth.C1()
+    o, r = c1.slice()
+    e = orc.compare(o.numpy(), r.numpy(), "f32", 1e-6, 1e-5, 60)
+    o, r = o.cuda(), r.cuda()
+    call = av.prepare(o, r, 1e-6, 1e-5, 60)
+    for _ in range(5):
+        assert_same(call(), e, "prepared")
+    e2 = orc.compare(o.cpu().numpy(), r.cpu().numpy(), "f32", 1e-6, 1e-5, 60, min_value=0.25, bounds=(-0.6, -0.4))
+    assert_same(av.prepare(o, r, 1e-6, 1e-5, 60, min_value=0.25, bounds=(-0.6, -0.4))(), e2, "prepared checks")
+
+
+def test_f32_index_beyond_2_pow_32(av):
+    """fp32 arrays of more than 2^32 elements: 64-bit indices through tiles, counts and report."""
+    n = (1 << 32) + 1000
+    ref = torch.zeros(n, dtype=torch.float32, device="cuda")
+    out = torch.zeros(n, dtype=torch.float32, device="cuda")
+    planted = [3, (1 << 32) - 2, (1 << 32) + 1, n - 1]
+    for i in planted:
+        out[i] = 1.0
+    g = av.compare(out, ref, 1e-6, 1e-5, 10)
+    assert g.n_mismatch == len(planted) and list(g.report["index"]) == planted
+    assert g.max_abs_err == 1.0 and g.max_rel_err == float("inf")
+    del out, ref
+    torch.cuda.empty_cache()

@@ -23,5 +23,10 @@ for n, label in ((1 << 20, "C1-size f32"), (1 << 26, "C2-size f32")):
         t2 = time.perf_counter()
         for _ in range(N): f(po, pr, n, 0, 1e-6, 1e-5, mr, br)
         t3 = time.perf_counter()
-        print(f"{label} mr={mr}: python compare {1e6*(t1-t0)/N:.1f} us/call, raw ctypes {1e6*(t3-t2)/N:.1f} us/call, kernels {1e3*ms/nl:.1f} us", flush=True)
+        call = av.prepare(o, r, 1e-6, 1e-5, mr, report=REP)
+        t4 = time.perf_counter()
+        for _ in range(N): call()
+        t5 = time.perf_counter()
+        print(f"{label} mr={mr}: python compare {1e6*(t1-t0)/N:.1f} us/call, prepared {1e6*(t5-t4)/N:.1f}, "
+              f"raw ctypes {1e6*(t3-t2)/N:.1f} us/call, kernels {1e3*ms/nl:.1f} us", flush=True)
 av.finalize()
