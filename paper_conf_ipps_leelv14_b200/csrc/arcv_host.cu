@@ -325,7 +325,7 @@ int wait_results(Ctx &c) {
     }
 }
 
-static int collect_timing(Ctx &c) {
+int collect_timing(Ctx &c) {
     if (c.n_ev) CK(cudaEventSynchronize(c.ev[c.n_ev - 1][1]));
     for (int i = 0; i < c.n_ev; ++i) {
         float ms = 0.f;
@@ -509,7 +509,7 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
         st = wait_results(c);
         if (st) return st;
     }
-    if (c.timing) {
+    if (c.timing && c.n_ev > Ctx::kMaxEv - 4) {  // read the event ring lazily: no per-call sync
         st = collect_timing(c);
         if (st) return st;
     }
@@ -712,6 +712,8 @@ int arc_verify_set_timing(int enable) {
 
 int arc_verify_kernel_stats(uint64_t *launches, double *total_ms, int reset) {
     if (!g_ctx) return ARC_E_NOINIT;
+    int st = collect_timing(*g_ctx);
+    if (st) return st;
     if (launches) *launches = g_ctx->timed_launches;
     if (total_ms) *total_ms = g_ctx->timed_ms;
     if (reset) {
