@@ -7,7 +7,7 @@ CUDA kernels.  ``compare`` / ``batch`` are conveniences over torch tensors
 (PyTorch is used for device memory, streams and process groups only).
 
 There is no CPU fallback: importing this package without the built library
-raises ImportError.  Build it with ``python -m paper_conf_ipps_leelv14_b200._build``
+raises ImportError.  Build it with ``python paper_conf_ipps_leelv14_b200/_build.py``
 or ``__graft_entry__.build()``.
 
 Paper: S. Lee, D. Li, J. S. Vetter, "Interactive Program Debugging and

@@ -13,9 +13,9 @@ HEADER = os.path.join(ROOT, "include", "arc_verify.h")
 
 @pytest.fixture(scope="module")
 def lib():
-    import paper_conf_ipps_leelv14_b200._build as b
+    from conftest import build_lib
 
-    b.build()
+    build_lib()
     import paper_conf_ipps_leelv14_b200 as av
 
     return av

@@ -6,9 +6,9 @@ import pytest
 
 @pytest.fixture(scope="module")
 def av():
-    import paper_conf_ipps_leelv14_b200._build as b
+    from conftest import build_lib
 
-    b.build()
+    build_lib()
     import paper_conf_ipps_leelv14_b200 as av
 
     return av
