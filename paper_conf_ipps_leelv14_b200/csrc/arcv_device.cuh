@@ -231,6 +231,15 @@ __device__ __forceinline__ uint64_t raw_bits(T v) {
     }
 }
 
+// Running maxima are order-independent, so a thread may adopt any value that
+// some thread of the same region has folded into its own maxima: the warp's
+// maxima are valid filter bounds for every lane (the fold is idempotent).
+// Called warp-uniformly.
+__device__ __forceinline__ void share_bounds(ThreadAcc &acc) {
+    acc.ma = warp_max_f64(acc.ma);
+    acc.rm = warp_max_f64(acc.rm);
+}
+
 // Seed the running maxima once per region per thread: evaluate exactly the
 // thread's element with the largest |x - y| and the one with the largest
 // (approximate) |x - y| / |y| in its first tile, so that the fast pass starts
@@ -264,22 +273,29 @@ __device__ __forceinline__ void seed_bounds(const uint8_t *so, const uint8_t *sr
     }
 }
 
-// Evaluate this thread's share of one tile; returns the mismatch bit mask
-// (bit k*EPV + j <-> tile element (k*256 + ctid)*EPV + j).  Floats: a fast pass
-// over all elements with the exact pre-filter, then the fp64 rule only for the
-// (rare) flagged elements, re-read from the still-held shared-memory stage.
+// Evaluate this thread's share of one tile; returns its number of mismatches
+// (K1 needs only counts; K2 re-derives the positions of the tiles it reports).
+// Thread element order: bit k*EPV + j <-> tile element (k*256 + ctid)*EPV + j.
+// Floats: a fast pass over all elements with the exact pre-filter, then the
+// fp64 rule only for the (rare) flagged elements, re-read from the still-held
+// shared-memory stage.
 template <typename T, bool kFull, bool kAligned>
-__device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *sr, uint32_t off_o, uint32_t off_r,
+__device__ __forceinline__ uint32_t eval_tile(const uint8_t *so, const uint8_t *sr, uint32_t off_o, uint32_t off_r,
                                               uint32_t cnt, int ctid, const SegHot &g, ThreadAcc &acc) {
     constexpr int EPV = 16 / sizeof(T);
     constexpr bool kFloat = std::is_floating_point<T>::value;
-    uint64_t mask = 0, slow = 0;
+    uint64_t slow = 0;
+    uint32_t nmis = 0;
     uint32_t bmax = 0;  // u8 only: byte-wise running max |a - b|
+    uint32_t dmax32 = 0;  // i32 only: running max |a - b| of this tile
     using RT = typename std::conditional<std::is_same<T, float>::value, float, double>::type;
     FastBounds<RT> fb;
     bool rel_form = true;
     if constexpr (kFloat) {
-        if (!acc.seeded) seed_bounds<T>(so, sr, off_o, off_r, cnt, ctid, g, acc);
+        if (!acc.seeded) {
+            seed_bounds<T>(so, sr, off_o, off_r, cnt, ctid, g, acc);
+            share_bounds(acc);
+        }
         if constexpr (std::is_same<T, float>::value) {
             refresh_bounds(acc, g.at_rd, g.rt_rd, fb);
             rel_form = g.rt_rd > 0.f;
@@ -319,13 +335,15 @@ __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *
                 const uint64_t m = int_absdiff<T>(xo[j], xr[j]);
                 if (m != 0 && (g.cflags & ARC_CHECK_VALUE_BOUNDS) && g.lo <= xv && xv <= g.hi) continue;
                 acc.imax = m > acc.imax ? m : acc.imax;
-                mis |= (uint32_t)(m != 0) << j;
+                mis += (uint32_t)(m != 0);
             }
-            mask |= (uint64_t)mis << (k * EPV);
+            nmis += mis;
         } else if constexpr (std::is_same<T, uint8_t>::value) {
-            // bytes: SIMD-within-a-register. |a-b| per byte (vabsdiffu4), running
-            // byte-wise max (vmaxu4), and 4 mismatch bits per word from vcmpne4.
-            uint32_t wa[4], wb[4], m16 = 0;
+            // bytes: SIMD-within-a-register.  |a-b| per byte is one native
+            // VABSDIFF4.U8; a byte mismatches iff its |a-b| is nonzero (bit 7 of
+            // each byte of nz); the byte-wise max (emulated vmaxu4) only runs for
+            // words that hold a mismatch.
+            uint32_t wa[4], wb[4];
             memcpy(wa, xo, 16);
             memcpy(wb, xr, 16);
 #pragma unroll
@@ -335,11 +353,11 @@ __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *
                     const uint32_t bm = ((vb * 0x00204081u) & 0x01010101u) * 0xffu;
                     wb[w] = (wb[w] & bm) | (wa[w] & ~bm);
                 }
-                const uint32_t ne = __vcmpne4(wa[w], wb[w]) & 0x01010101u;
-                m16 |= ((ne * 0x10204080u) >> 28) << (4 * w);  // byte i -> bit i
-                bmax = __vmaxu4(bmax, __vabsdiffu4(wa[w], wb[w]));
+                const uint32_t ad = __vabsdiffu4(wa[w], wb[w]);
+                const uint32_t nz = (((ad & 0x7f7f7f7fu) + 0x7f7f7f7fu) | ad) & 0x80808080u;
+                nmis += __popc(nz);
+                if (ad != 0u) bmax = __vmaxu4(bmax, ad);
             }
-            mask |= (uint64_t)(m16 & valid) << (k * EPV);
         } else if constexpr (kFloat) {
             uint32_t sl = 0;
             if (rel_form) {
@@ -350,17 +368,30 @@ __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *
                 for (int j = 0; j < EPV; ++j) sl |= (uint32_t)(!fast_ok<false>((RT)xo[j], (RT)xr[j], fb)) << j;
             }
             slow |= (uint64_t)(sl & valid) << (k * EPV);
+        } else if constexpr (sizeof(T) == 4) {
+            // int32: |a - b| <= 2^32 - 1 is exact in 32-bit unsigned arithmetic
+            // (sad.s32 wraps mod 2^32); a per-tile 32-bit running max, folded
+            // into the 64-bit accumulator once per tile.
+            uint32_t mis = 0;
+#pragma unroll
+            for (int j = 0; j < EPV; ++j) {
+                const uint32_t m = ((valid >> j) & 1u) ? __sad((int)xo[j], (int)xr[j], 0u) : 0u;
+                dmax32 = max(dmax32, m);
+                mis += min(m, 1u);
+            }
+            nmis += mis;
         } else {
             uint32_t mis = 0;
 #pragma unroll
             for (int j = 0; j < EPV; ++j) {
                 const uint64_t m = ((valid >> j) & 1u) ? int_absdiff<T>(xo[j], xr[j]) : 0ull;
                 acc.imax = m > acc.imax ? m : acc.imax;
-                mis |= (uint32_t)(m != 0) << j;
+                mis += (uint32_t)(m != 0);
             }
-            mask |= (uint64_t)mis << (k * EPV);
+            nmis += mis;
         }
     }
+    if constexpr (!kFloat && sizeof(T) == 4) acc.imax = (uint64_t)dmax32 > acc.imax ? (uint64_t)dmax32 : acc.imax;
     if constexpr (std::is_same<T, uint8_t>::value) {
         const uint32_t m2 = __vmaxu4(bmax, bmax >> 16);
         const uint64_t mb = (uint64_t)max(m2 & 0xffu, (m2 >> 8) & 0xffu);
@@ -378,17 +409,20 @@ __device__ __forceinline__ uint64_t eval_tile(const uint8_t *so, const uint8_t *
                 // the bounds grew since the fast pass: a re-check clears most of a
                 // warm-up tile's flags without the fp64 rule
                 if (rel_form ? fast_ok<true>((RT)x, (RT)y, fb) : fast_ok<false>((RT)x, (RT)y, fb)) continue;
-                mask |= (uint64_t)eval_f64_checked((double)x, (double)y, g, acc) << b;
+                nmis += (uint32_t)eval_f64_checked((double)x, (double)y, g, acc);
                 if constexpr (std::is_same<T, float>::value) refresh_bounds(acc, g.at_rd, g.rt_rd, fb);
                 else refresh_bounds(acc, g.abs_tol, g.rel_tol, fb);
             }
         }
+        // a lane's new maxima become the whole warp's filter bounds (the warp
+        // then meets ~ln(32 n) record-breaking elements instead of ~ln(n) per lane)
+        if (__any_sync(0xffffffffu, slow != 0)) share_bounds(acc);
     }
-    return mask;
+    return nmis;
 }
 
 template <typename T>
-__device__ __forceinline__ uint64_t eval_tile_dispatch(const uint8_t *so, const uint8_t *sr, const StageInfo &si,
+__device__ __forceinline__ uint32_t eval_tile_dispatch(const uint8_t *so, const uint8_t *sr, const StageInfo &si,
                                                        int ctid, const SegHot &g, ThreadAcc &acc) {
     constexpr uint32_t TE = kTileBytes / sizeof(T);
     const bool full = si.count == TE;
@@ -401,7 +435,7 @@ __device__ __forceinline__ uint64_t eval_tile_dispatch(const uint8_t *so, const 
     return eval_tile<T, false, false>(so, sr, si.off_o, si.off_r, si.count, ctid, g, acc);
 }
 
-__device__ __forceinline__ uint64_t eval_any(const uint8_t *so, const uint8_t *sr, const StageInfo &si, int ctid,
+__device__ __forceinline__ uint32_t eval_any(const uint8_t *so, const uint8_t *sr, const StageInfo &si, int ctid,
                                              const SegHot &g, ThreadAcc &acc) {
     switch (g.dtype) {
         case ARC_F32: return eval_tile_dispatch<float>(so, sr, si, ctid, g, acc);
@@ -606,8 +640,7 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
             g.load(segs[si.seg]);
         }
         const uint8_t *so = smem + (size_t)s * kStageBytes;
-        const uint64_t mask = (p.flags & kFlagProbe) ? 0ull : eval_any(so, so + kStageArrayBytes, si, ctid, g, acc);
-        const uint32_t cnt = (uint32_t)__popcll(mask);
+        const uint32_t cnt = (p.flags & kFlagProbe) ? 0u : eval_any(so, so + kStageArrayBytes, si, ctid, g, acc);
         acc.count += cnt;
         if (g.max_report != 0) {
             // Per-tile count for K2: warps fold their counts into the stage's

@@ -288,7 +288,7 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
     if (need_compact) {
         p.finalize = finalize ? 1 : 0;
         p.done_base = c.done_base;
-        const uint32_t grid2 = (uint32_t)c.num_sms;
+        const uint32_t grid2 = (uint32_t)c.k2_grid;
         void *args[] = {&p};
         e = cudaLaunchCooperativeKernel((const void *)arcv_compact_kernel, dim3(grid2), dim3(kConsumerThreads), args,
                                         kCompactSmem, c.stream);
@@ -623,13 +623,19 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
     int occ = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kf, kThreads, smem));
     if (occ < 1) { set_error("kernel does not fit on an SM (smem %zu)", smem); return ARC_E_UNSUPPORTED; }
+    // K2: as many co-resident CTAs as fit (cooperative launch), so the re-read
+    // tiles of a sparse report are all in flight in one wave
+    int occ2 = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, arcv_compact_kernel, kConsumerThreads, kCompactSmem));
+    const int k2cap = env_int("ARCV_K2_PER_SM", 2);
+    c->k2_grid = c->num_sms * std::max(1, std::min(occ2, k2cap > 0 ? k2cap : 1));
     const int cap = env_int("ARCV_CTAS_PER_SM", 0);
     c->ctas_per_sm = cap > 0 ? std::min(cap, occ) : occ;
     if (env_int("ARCV_VERBOSE", 0)) {
         cudaFuncAttributes fa;
         CK(cudaFuncGetAttributes(&fa, kf));
-        fprintf(stderr, "[arcv] sms=%d stages=%d ctas/sm=%d (occupancy %d) regs=%d static_smem=%zu dyn_smem=%zu local=%zu\n",
-                c->num_sms, c->stages, c->ctas_per_sm, occ, fa.numRegs, fa.sharedSizeBytes, smem, fa.localSizeBytes);
+        fprintf(stderr, "[arcv] sms=%d stages=%d ctas/sm=%d (occupancy %d) k2_grid=%d regs=%d static_smem=%zu dyn_smem=%zu local=%zu\n",
+                c->num_sms, c->stages, c->ctas_per_sm, occ, c->k2_grid, fa.numRegs, fa.sharedSizeBytes, smem, fa.localSizeBytes);
     }
     // counters: [0] tile tickets, [1] finished CTAs, [2] K2 grid barrier,
     // [3] 2 x u32 active-list lengths, [4] 2 x u32 pool lengths (by parity)

@@ -20,6 +20,7 @@ struct Ctx {
     int rank = 0, nranks = 1;
     bool sharded = false;  // collective path (NCCL communicator), nranks >= 1
     int num_sms = 0, ctas_per_sm = 1, stages = 3, flags = 0;
+    int k2_grid = 0;  // K2 (cooperative) grid: SMs x co-resident CTAs (<= 2)
     cudaStream_t stream = nullptr;
     bool own_stream = false;
     cudaStream_t copy_stream = nullptr;

@@ -20,34 +20,11 @@
 
 #include "arc_verify.h"
 #include "arcv_internal.h"
+#include "arcv_merge.h"
 
 namespace arcv {
 
 constexpr uint64_t kPacketEntries = 4096;  // K: entries carried in the all-gather
-constexpr int kMaxRanks = 256;
-
-// ------------------------------------------------------------- merge plan
-// Shared by the host entry point and the merge kernel (one definition).
-__host__ __device__ inline void merge_plan_impl(const arc_shard_header_t *h, int p, uint64_t max_report,
-                                                arc_shard_plan_t *plan, arc_shard_header_t *g) {
-    uint64_t off = 0, pre = 0;
-    g->n = 0;
-    g->n_mismatch = 0;
-    g->max_abs_bits = 0;
-    g->max_rel_bits = 0;
-    for (int r = 0; r < p; ++r) {
-        plan[r].index_offset = off;
-        plan[r].prefix = pre;
-        const uint64_t rem = max_report > pre ? max_report - pre : 0;
-        plan[r].contrib = h[r].n_mismatch < rem ? h[r].n_mismatch : rem;
-        off += h[r].n;
-        pre += h[r].n_mismatch;
-        g->n += h[r].n;
-        g->n_mismatch += h[r].n_mismatch;
-        g->max_abs_bits = h[r].max_abs_bits > g->max_abs_bits ? h[r].max_abs_bits : g->max_abs_bits;
-        g->max_rel_bits = h[r].max_rel_bits > g->max_rel_bits ? h[r].max_rel_bits : g->max_rel_bits;
-    }
-}
 
 // Every block rebuilds the plan in shared memory (p <= 256 headers), then the
 // grid copies the packet entries that belong to the global report, adding each

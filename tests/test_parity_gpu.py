@@ -139,6 +139,28 @@ def test_all_mismatch_and_report_limits(av, orc, dt):
         run_both(av, orc, out, ref, dt, 0.0, 0.0, mr, f"all-mismatch {dt} mr={mr}")
 
 
+@pytest.mark.parametrize("dt", ["i32", "i64"])
+def test_integer_extremes(av, orc, dt):
+    """|a - b| at the ends of the range (i32: up to 2^32 - 1, exact in the 32-bit
+    path; i64: up to 2^64 - 1, rounded to double) -- reading R9."""
+    info = np.iinfo(NP[dt])
+    lo, hi = int(info.min), int(info.max)
+    vals = [lo, lo + 1, -1, 0, 1, hi - 1, hi]
+    pairs = [(a, b) for a in vals for b in vals]
+    n = 3 * TILE_ELEMS[dt] + 5  # several tiles and a ragged tail; extremes in every tile
+    gen = np.random.default_rng(11)
+    ref = gen.integers(lo, hi, size=n, dtype=NP[dt], endpoint=True)
+    out = ref.copy()
+    for t in range(4):
+        for k, (a, b) in enumerate(pairs):
+            i = min(n - 1, t * TILE_ELEMS[dt] + 3 * k)
+            out[i], ref[i] = a, b
+    o, r = torch.from_numpy(out).cuda(), torch.from_numpy(ref).cuda()
+    for mr in (0, 7, 10 ** 6):
+        g, _ = run_both(av, orc, o, r, dt, 0, 0, mr, f"{dt} extremes mr={mr}")
+    assert g.max_abs_err == float(hi - lo)
+
+
 def test_aliasing(av, orc):
     c1 = synth.C1()
     out, _ = c1.slice()

@@ -1,0 +1,208 @@
+"""A/B of library builds on the same box: python tools/ab.py LIB_A.so LIB_B.so [...]
+
+Each library is loaded with its own ctypes handle (distinct file names give
+distinct copies of the library's static context), initialised on torch's
+stream, and run on the same HBM-resident workloads in alternating rounds.
+Prints per workload and library: median kernel time (the library's CUDA
+events around K1+K2) and median wall time per call, and checks that every
+library returns the identical summary + report.
+"""
+import ctypes
+import os
+import statistics
+import sys
+import time
+
+sys.path.insert(0, os.getcwd())
+import numpy as np
+import torch
+
+import paper_conf_ipps_leelv14_b200 as av
+import synth
+
+libs = sys.argv[1:] or [av.LIB_PATH]
+ROUNDS = int(os.environ.get("AB_ROUNDS", "3"))
+STEPS = int(os.environ.get("AB_STEPS", "20"))
+ONLY = os.environ.get("AB_ONLY")
+
+
+def load(path):
+    lib = ctypes.CDLL(os.path.abspath(path))
+    P, U64, I, D = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int, ctypes.c_double
+    lib.arc_verify_init.argtypes = [ctypes.POINTER(av.arc_verify_opts_t)]
+    lib.arc_verify_compare.argtypes = [P, P, U64, I, D, D, U64, ctypes.POINTER(av.arc_verify_result_t)]
+    lib.arc_verify_batch.argtypes = [ctypes.POINTER(av.arc_verify_region_t), ctypes.c_size_t,
+                                     ctypes.POINTER(av.arc_verify_result_t)]
+    lib.arc_verify_set_timing.argtypes = [I]
+    lib.arc_verify_kernel_stats.argtypes = [ctypes.POINTER(U64), ctypes.POINTER(D), I]
+    lib.arc_verify_last_error.restype = ctypes.c_char_p
+    return lib
+
+
+torch.cuda.set_device(0)
+stream = torch.cuda.current_stream().cuda_stream or av.CUDA_STREAM_LEGACY
+L = []
+for p in libs:
+    lib = load(p)
+    opts = av.arc_verify_opts_t(0, stream, 0, 1, None)
+    assert lib.arc_verify_init(ctypes.byref(opts)) == 0, lib.arc_verify_last_error()
+    L.append(lib)
+
+REP = [torch.empty(24 * (1 << 20), dtype=torch.uint8, pin_memory=True).numpy().view(av.REPORT_DTYPE)
+       for _ in L]
+
+
+def single(o, r, at, rt, mr):
+    code = av.dtype_code(o)
+    n = o.numel()
+
+    def mk(k):
+        res = av.arc_verify_result_t()
+        res.report = REP[k].ctypes.data
+        f, br, po, pr = L[k].arc_verify_compare, ctypes.byref(res), o.data_ptr(), r.data_ptr()
+
+        def call():
+            st = f(po, pr, n, code, at, rt, mr, br)
+            assert st == 0, L[k].arc_verify_last_error()
+
+        def result():
+            return (res.n_mismatch, res.max_abs_err, res.max_rel_err, res.n_reported,
+                    bytes(REP[k][:res.n_reported].tobytes()))
+        return call, result
+    return mk, 2 * n * o.element_size()
+
+
+def batch(pairs):
+    nb = 0
+    for (o, r, at, rt, mr) in pairs:
+        nb += 2 * o.numel() * o.element_size()
+
+    def mk(k):
+        R = (av.arc_verify_region_t * len(pairs))()
+        res = (av.arc_verify_result_t * len(pairs))()
+        off = 0
+        reps = []
+        for i, (o, r, at, rt, mr) in enumerate(pairs):
+            R[i].out, R[i].ref, R[i].n = o.data_ptr(), r.data_ptr(), o.numel()
+            R[i].dtype, R[i].abs_tol, R[i].rel_tol, R[i].max_report = av.dtype_code(o), at, rt, mr
+            res[i].report = REP[k][off:].ctypes.data
+            reps.append((off, i))
+            off += mr
+
+        def call():
+            st = L[k].arc_verify_batch(R, len(pairs), res)
+            assert st == 0, L[k].arc_verify_last_error()
+
+        def result():
+            return tuple((res[i].n_mismatch, res[i].max_abs_err, res[i].max_rel_err, res[i].n_reported,
+                          bytes(REP[k][o_:o_ + res[i].n_reported].tobytes())) for (o_, i) in reps)
+        return call, result
+    return mk, nb
+
+
+W = {}
+
+
+def add(name, fn):
+    if ONLY and name not in ONLY.split(","):
+        return
+    W[name] = fn
+
+
+def c1():
+    o, r = synth.C1().slice(device="cuda")
+    return single(o, r, 1e-6, 1e-5, 1 << 20)
+
+
+def c2(v):
+    def f():
+        o, r = synth.C2(v).slice(device="cuda")
+        return single(o, r, 0.0, 1e-5, 1 << 20)
+    return f
+
+
+def f32u():
+    reg = synth.configs.Region("F", "f32", 1 << 26, 77, 1e-6, 1e-5, 1 << 20, "f32")
+    o, r = reg.slice(device="cuda")
+    return single(o, r, 1e-6, 1e-5, 1 << 20)
+
+
+def c3():
+    pairs = []
+    for reg in synth.c3_regions():
+        o, r = reg.slice(device="cuda")
+        pairs.append((o, r, reg.abs_tol, reg.rel_tol, reg.max_report))
+    return batch(pairs)
+
+
+def c4():
+    c = synth.C4()
+    o, r = c.slice(device="cuda")
+    return single(o, r, c.abs_tol, c.rel_tol, c.max_report)
+
+
+def i32clean():
+    reg = synth.configs.Region("I", "i32", 1 << 28, 78, 0, 0, 1 << 20, "i32")
+    o, r = reg.slice(device="cuda")
+    return single(o, r, 0, 0, 1 << 20)
+
+
+def u8clean():
+    reg = synth.configs.Region("I", "i32", 1 << 28, 78, 0, 0, 1 << 20, "i32")
+    o, r = reg.slice(device="cuda")
+    return single(o.view(torch.uint8), r.view(torch.uint8), 0, 0, 1 << 20)
+
+
+def c5():
+    c = synth.C5()
+    o, r = c.slice(device="cuda")
+    return single(o, r, 0, 0, c.max_report)
+
+
+add("C1", c1)
+add("C2A", c2("A"))
+add("C2B", c2("B"))
+add("f32u_2^26", f32u)
+add("C3batch", c3)
+add("i32clean_2^28", i32clean)
+add("u8clean_2^30", u8clean)
+add("C4", c4)
+add("C5", c5)
+
+print(f"libs: {libs}; rounds {ROUNDS} x {STEPS} steps", flush=True)
+for name, make in W.items():
+    mk, nbytes = make()
+    calls = [mk(k) for k in range(len(L))]
+    ref_res = None
+    kern = [[] for _ in L]
+    wall = [[] for _ in L]
+    for k, (call, result) in enumerate(calls):
+        for _ in range(3):
+            call()
+        res = result()
+        if ref_res is None:
+            ref_res = res
+        assert res == ref_res, f"{name}: lib {libs[k]} result differs"
+    torch.cuda.synchronize()
+    for rd in range(ROUNDS):
+        for k, (call, _r) in enumerate(calls):
+            lib = L[k]
+            lib.arc_verify_set_timing(1)
+            n_, ms_ = ctypes.c_uint64(), ctypes.c_double()
+            lib.arc_verify_kernel_stats(ctypes.byref(n_), ctypes.byref(ms_), 1)
+            t0 = time.perf_counter()
+            for _ in range(STEPS):
+                call()
+            t1 = time.perf_counter()
+            lib.arc_verify_kernel_stats(ctypes.byref(n_), ctypes.byref(ms_), 1)
+            lib.arc_verify_set_timing(0)
+            kern[k].append(1e3 * ms_.value / max(n_.value, 1))
+            wall[k].append(1e6 * (t1 - t0) / STEPS)
+    line = [f"{name:14s} {nbytes / 2**20:9.1f} MiB"]
+    for k in range(len(L)):
+        km, wm = statistics.median(kern[k]), statistics.median(wall[k])
+        line.append(f"| {os.path.basename(libs[k])[:18]:18s} kern {km:8.1f} us {nbytes / km / 1e3:7.1f} GB/s"
+                    f"  call {wm:8.1f} us {nbytes / wm / 1e3:7.1f} GB/s")
+    print(" ".join(line), flush=True)
+    del calls, mk
+    torch.cuda.empty_cache()
