@@ -87,7 +87,8 @@ typedef struct {
     double max_abs_err;     /* max defined d; 0 for empty / all-NaN                 */
     double max_rel_err;     /* max defined r; 0 for integer dtypes                  */
     uint64_t n_reported;    /* = min(n_mismatch, max_report)                        */
-    arc_mismatch_t *report; /* CALLER-owned, capacity >= min(max_report, n) entries;
+    arc_mismatch_t *report; /* CALLER-owned, capacity >= min(max_report, n) entries
+                               (sharded: the GLOBAL n);
                                host memory (pageable or pinned) or device memory on
                                the library's device (then nothing crosses PCIe)     */
 } arc_verify_result_t;
@@ -98,9 +99,11 @@ typedef struct {
                                    non-blocking stream (the caller orders its own work);
                                    (void*)1 = cudaStreamLegacy, the legacy default stream */
     int rank, nranks;           /* sharded mode when nranks > 1                           */
-    const void *nccl_unique_id; /* 128-byte ncclUniqueId (same on all ranks); required if
-                                   nranks > 1; with nranks == 1 it selects the collective
-                                   path over a 1-rank communicator                        */
+    const void *nccl_unique_id; /* 128-byte ncclUniqueId (same on all ranks), or NULL.
+                                   nranks > 1 needs it, or the peer windows
+                                   (arc_verify_peer_export / _open), or both; with
+                                   nranks == 1 an id selects the collective path over a
+                                   1-rank communicator                                    */
 } arc_verify_opts_t;
 
 /*
@@ -137,12 +140,14 @@ typedef struct {
 /*
  * arc_verify_init -- create the process context.
  *   opts == NULL: device 0, library-owned stream, one rank.
- *   nranks > 1: sharded mode; nccl_unique_id must be the id produced by
- *   arc_verify_get_unique_id on one rank and shared with all ranks; NCCL
- *   (libnccl.so.2, the one already loaded by the process if any) is opened
- *   at run time.
- * Errors: ARC_E_INVAL (bad device / rank / nranks, missing id), ARC_E_CUDA,
- * ARC_E_NCCL.  Calling init twice without finalize returns ARC_E_INVAL.
+ *   nranks > 1: sharded mode.  The exchange runs over the peer windows when
+ *   they are open (arc_verify_peer_export + arc_verify_peer_open, below), else
+ *   over NCCL: nccl_unique_id is then the id produced by
+ *   arc_verify_get_unique_id on one rank and shared with all ranks, and NCCL
+ *   (libnccl.so.2, the one already loaded by the process if any) is opened at
+ *   run time.
+ * Errors: ARC_E_INVAL (bad device / rank / nranks), ARC_E_CUDA, ARC_E_NCCL.
+ * Calling init twice without finalize returns ARC_E_INVAL.
  */
 int arc_verify_init(const arc_verify_opts_t *opts);
 
@@ -331,6 +336,34 @@ int arc_verify_shard_local(const void *out, const void *ref, uint64_t n, arc_dty
  */
 int arc_verify_shard_merge(const void *gathered_dev, int nranks, uint64_t packet_entries, uint64_t max_report,
                            arc_verify_result_t *result);
+
+/* ------------------------------------------------------------------------
+ * Peer-memory exchange (the B200 path of step a8).
+ * Each rank owns a "window" in its HBM -- 2 x 256 flag words and two packets
+ * (call parities) of {32-byte header, max_report_cap entries} -- mapped into
+ * every other rank through CUDA IPC (NVLink / NVSwitch peer memory).  A
+ * sharded arc_verify_compare with max_report <= max_report_cap then runs
+ * local compare -> ONE exchange kernel (publish header + flags with
+ * system-scope release stores into every window, wait for all flags, merge by
+ * reading the peers' packets directly) -> one host wait; no NCCL call.
+ * Setup is collective: every rank calls arc_verify_peer_export, the caller
+ * all-gathers the 64-byte handles in rank order (e.g. torch.distributed), and
+ * every rank calls arc_verify_peer_open.  All ranks must use the same
+ * max_report_cap.  Ranks on the same GPU (different processes) work too.
+ * ------------------------------------------------------------------------ */
+
+/* Allocate this rank's window for reports of up to max_report_cap entries
+ * (2 * (32 + 24 * cap) bytes + 4 KiB of flags, zeroed) and write its 64-byte
+ * cudaIpcMemHandle_t to `handle`.  Re-exporting replaces the window (peers must
+ * re-open).  Errors: ARC_E_NOINIT, ARC_E_INVAL (NULL handle, cap > 2^36),
+ * ARC_E_NOMEM, ARC_E_CUDA. */
+int arc_verify_peer_export(uint64_t max_report_cap, void *handle);
+
+/* Map the peers' windows: `handles` = nranks x 64 bytes in rank order (the
+ * own entry is ignored).  Enables the peer path.  Errors: ARC_E_NOINIT,
+ * ARC_E_INVAL (no export yet, NULL handles), ARC_E_UNSUPPORTED (a handle cannot
+ * be mapped, e.g. no P2P between the devices; the NCCL path stays in use). */
+int arc_verify_peer_open(const void *handles);
 
 #ifdef __cplusplus
 }

@@ -39,6 +39,7 @@ EXPORTED = [
     "arc_verify_version", "arc_verify_merge_plan", "arc_verify_packet_bytes",
     "arc_verify_shard_local", "arc_verify_shard_merge", "arc_verify_probe_read", "arc_verify_compare_ex",
     "arc_verify_checksum", "arc_verify_selected", "arc_verify_batch_selected", "arc_verify_format_result",
+    "arc_verify_peer_export", "arc_verify_peer_open",
 ]
 
 
@@ -120,6 +121,8 @@ def _load() -> ctypes.CDLL:
                                           ctypes.POINTER(arc_verify_result_t), P]),
         "arc_verify_format_result": (I, [ctypes.c_char_p, I, D, D, ctypes.POINTER(arc_verify_result_t), U64,
                                          ctypes.c_char_p, SZ]),
+        "arc_verify_peer_export": (I, [U64, P]),
+        "arc_verify_peer_open": (I, [P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -218,6 +221,20 @@ def arc_verify_shard_merge(gathered_ptr, nranks, packet_entries, max_report, res
            "arc_verify_shard_merge")
 
 
+def arc_verify_peer_export(max_report_cap: int) -> bytes:
+    """Allocate this rank's exchange window; returns its 64-byte IPC handle."""
+    buf = ctypes.create_string_buffer(64)
+    _check(_lib.arc_verify_peer_export(max_report_cap, buf), "arc_verify_peer_export")
+    return buf.raw
+
+
+def arc_verify_peer_open(handles: Sequence[bytes]) -> None:
+    """Map every rank's window (handles in rank order) and enable the peer path."""
+    blob = b"".join(bytes(h) for h in handles)
+    buf = ctypes.create_string_buffer(blob, len(blob))
+    _check(_lib.arc_verify_peer_open(buf), "arc_verify_peer_open")
+
+
 def arc_verify_probe_read(a_ptr: int, b_ptr: int, nbytes: int, iters: int = 10) -> float:
     """Diagnostic: read-only streaming GB/s of the comparison's pipeline (no predicate)."""
     g = ctypes.c_double()
@@ -294,7 +311,7 @@ def dtype_code(t) -> int:
         raise TypeError(f"unsupported dtype {t.dtype}") from None
 
 
-_state = {"init": False}
+_state = {"init": False, "nranks": 1}
 
 
 def init(device: Optional[int] = None, stream=None, rank: int = 0, nranks: int = 1,
@@ -311,23 +328,59 @@ def init(device: Optional[int] = None, stream=None, rank: int = 0, nranks: int =
         handle = CUDA_STREAM_LEGACY  # torch's default stream is the legacy NULL stream
     arc_verify_init(device, handle, rank, nranks, nccl_unique_id)
     _state["init"] = True
+    _state["nranks"] = nranks
 
 
-def init_distributed(group=None) -> None:
-    """Sharded init over a torch.distributed group: rank 0 creates the NCCL id."""
+def init_distributed(group=None, transport: str = "peer", max_report_cap: int = 1 << 20) -> str:
+    """Sharded init over a torch.distributed group (any backend; only small host
+    objects travel through it).  Returns the exchange in use.
+
+    transport="peer": peer-memory windows only (CUDA IPC over NVLink; also ranks
+        sharing one GPU) -- the device-driven exchange, no NCCL.
+    transport="nccl": NCCL communicator only (rank 0 creates the id).
+    transport="auto": both; compares use the windows when max_report <=
+        max_report_cap and fall back to NCCL otherwise (or if mapping fails).
+    """
     import torch
     import torch.distributed as dist
 
+    if transport not in ("peer", "nccl", "auto"):
+        raise ValueError(f"unknown transport {transport!r}")
     rank, world = dist.get_rank(group), dist.get_world_size(group)
-    obj = [arc_verify_get_unique_id() if rank == 0 else None]
-    dist.broadcast_object_list(obj, src=0, group=group)
-    init(torch.cuda.current_device(), None, rank, world, obj[0])
+    uid = None
+    if transport in ("nccl", "auto"):
+        obj = [arc_verify_get_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0, group=group)
+        uid = obj[0]
+    init(torch.cuda.current_device(), None, rank, world, uid)
+    if transport == "nccl":
+        return "nccl"
+    h = arc_verify_peer_export(max_report_cap)
+    handles = [None] * world
+    dist.all_gather_object(handles, h, group=group)
+    try:
+        arc_verify_peer_open(handles)
+        ok = 1
+    except ArcVerifyError:
+        if transport == "peer":
+            raise
+        ok = 0
+    # every rank must take the same path: agree on the outcome
+    flags = [None] * world
+    dist.all_gather_object(flags, ok, group=group)
+    if not all(flags):
+        if transport == "peer":
+            raise RuntimeError("peer windows could not be mapped on every rank")
+        arc_verify_peer_export(0)  # drops the windows: the peer path stays off, NCCL is used
+        return "nccl"
+    return "peer"
 
 
 def finalize() -> None:
     if _state["init"]:
         arc_verify_finalize()
         _state["init"] = False
+        _state["nranks"] = 1
 
 
 def _report_buffer(cap: int):
@@ -375,7 +428,8 @@ def compare(out, ref, abs_tol: float = 0.0, rel_tol: float = 0.0, max_report: in
     if n and not (out.is_contiguous() and ref.is_contiguous()):
         raise ValueError("tensors must be contiguous")
     if report is None:
-        rep_arr, rep_ptr = _report_buffer(min(int(max_report), n))
+        # sharded: the global report may exceed the local shard's length
+        rep_arr, rep_ptr = _report_buffer(int(max_report) if _state["nranks"] > 1 else min(int(max_report), n))
     elif isinstance(report, np.ndarray):
         rep_arr, rep_ptr = report, report.ctypes.data
     else:
@@ -422,7 +476,7 @@ class Prepared:
         if n and not (out.is_contiguous() and ref.is_contiguous()):
             raise ValueError("tensors must be contiguous")
         if report is None:
-            report, ptr = _report_buffer(min(int(max_report), n))
+            report, ptr = _report_buffer(int(max_report) if _state["nranks"] > 1 else min(int(max_report), n))
         elif isinstance(report, np.ndarray):
             ptr = report.ctypes.data
         else:

@@ -542,6 +542,7 @@ __device__ __forceinline__ void finalize_launch(const Params &p, int tid, int nt
             a.max_rel_bits = __ldcg(&p.acc[k].max_rel_bits);
             a.pad = 0;
             p.result[k] = a;
+            if (p.mirror) p.mirror[k] = a;
             p.acc[k].count = 0;
             p.acc[k].max_abs_bits = 0;
             p.acc[k].max_rel_bits = 0;

@@ -271,6 +271,7 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
     p.flags = (uint32_t)c.flags;
     p.done_flag = (c.flags & 8) ? nullptr : c.flag_dev;  // ARCV_FLAGS bit 3 (diagnostic): stream sync
     if (finalize) p.seq = ++c.seq;  // the host waits for the last finalize launch's number
+    p.mirror = finalize ? c.mirror_next : nullptr;
     for (uint32_t k = 0; k < n_segs; ++k)
         if (segs[k].report && classify(segs[k].report, c.device) != PK_DEVICE) p.report_host = 1;
 
@@ -504,6 +505,7 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
                            slot_of[k]);
         if (st) return st;
     }
+    if (c.defer_wait) return ARC_OK;  // the peer-exchange kernel reads the mirror
     const uint32_t n_slots = next_slot;
     if (n_slots) {  // result slots are mapped host memory
         st = wait_results(c);
@@ -573,9 +575,10 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
     o.nranks = 1;
     if (opts) o = *opts;
     if (o.nranks < 1 || o.rank < 0 || o.rank >= o.nranks) { set_error("bad rank/nranks"); return ARC_E_INVAL; }
-    if (o.nranks > 1 && !o.nccl_unique_id) { set_error("nranks > 1 needs nccl_unique_id"); return ARC_E_INVAL; }
-    // an NCCL id selects the collective path even for one rank (a 1-rank
-    // communicator), which lets a single GPU exercise it end to end
+    // nranks > 1 without an NCCL id: peer-memory exchange only (arc_verify_peer_*
+    // must be called before the first collective compare).  An NCCL id selects
+    // the collective path even for one rank (a 1-rank communicator), which lets
+    // a single GPU exercise it end to end.
     int ndev = 0;
     cudaError_t e = cudaGetDeviceCount(&ndev);
     if (e != cudaSuccess) { cudaGetLastError(); return cuda_fail(e, "cudaGetDeviceCount"); }
@@ -652,8 +655,8 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
     if (e != cudaSuccess) { cudaGetLastError(); set_error("cudaMalloc pool list"); return ARC_E_NOMEM; }
     CK(cudaStreamSynchronize(c->stream));
     g_ctx = c;
-    c->sharded = o.nccl_unique_id != nullptr;
-    if (c->sharded) {
+    c->sharded = o.nccl_unique_id != nullptr || o.nranks > 1;
+    if (o.nccl_unique_id) {
         int st = shard_init(*c, o.nccl_unique_id);
         if (st) {
             arc_verify_finalize();
@@ -667,6 +670,7 @@ int arc_verify_finalize(void) {
     if (!g_ctx) return ARC_E_NOINIT;
     Ctx *c = g_ctx;
     cudaStreamSynchronize(c->stream);
+    peer_finalize(*c);
     shard_finalize(*c);
     cudaFree(c->counters);
     cudaFree(c->tile_cnt);

@@ -5,6 +5,7 @@
 #include <cstdint>
 
 #include "arc_verify.h"
+#include "arcv_merge.h"
 #include "arcv_types.h"
 
 namespace arcv {
@@ -64,6 +65,20 @@ struct Ctx {
     uint8_t *gathered = nullptr;       size_t gathered_cap = 0;   // bytes
     arc_shard_header_t *hdr_host = nullptr; size_t hdr_host_cap = 0;
     arc_shard_header_t *merge_dev = nullptr;                        // [1 + nranks] global + per-rank
+
+    // peer-memory exchange (arcv_peer.cu): symmetric windows over NVLink P2P
+    bool defer_wait = false;           // run_local: enqueue only (the exchange kernel follows)
+    Acc *mirror_next = nullptr;        // launch_segments: device copy of the finalised slots
+    Acc *mirror = nullptr;             // [1] device
+    uint8_t *win = nullptr;            // own window (cudaMalloc, IPC-exported)
+    size_t win_bytes = 0;
+    uint64_t win_cap = 0;              // report entries per packet
+    void *peer_map[kMaxRanks] = {};    // IPC-mapped peer windows (to close)
+    uint8_t **win_table = nullptr;     // device [nranks] window pointers (own included)
+    bool peer_ready = false;
+    unsigned long long coll_seq = 0;   // collective calls made (flag value of the last)
+    unsigned long long peer_done_base = 0;
+    arc_shard_header_t *peer_out_host = nullptr, *peer_out_dev = nullptr;  // mapped [2]: global, status
 };
 
 extern Ctx *g_ctx;
@@ -82,5 +97,11 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
 int shard_init(Ctx &c, const void *nccl_unique_id);
 void shard_finalize(Ctx &c);
 int shard_compare(Ctx &c, const arc_verify_region_t &r, arc_verify_result_t *result);
+int report_target(Ctx &c, arc_verify_result_t *result, uint64_t cap, arc_mismatch_t **dst, bool *host);
+void fill_result(const arc_shard_header_t &g, uint64_t max_report, arc_verify_result_t *res);
+
+// arcv_peer.cu
+int peer_compare(Ctx &c, const arc_verify_region_t &r, arc_verify_result_t *result);
+void peer_finalize(Ctx &c);
 
 }  // namespace arcv

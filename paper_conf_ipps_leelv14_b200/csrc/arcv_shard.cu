@@ -224,7 +224,7 @@ static int merge_gathered(Ctx &c, const uint8_t *gathered, int p, uint64_t K, ui
     return ARC_OK;
 }
 
-static void fill_result(const arc_shard_header_t &g, uint64_t max_report, arc_verify_result_t *res) {
+void fill_result(const arc_shard_header_t &g, uint64_t max_report, arc_verify_result_t *res) {
     res->n = g.n;
     res->n_mismatch = g.n_mismatch;
     memcpy(&res->max_abs_err, &g.max_abs_bits, 8);
@@ -233,7 +233,7 @@ static void fill_result(const arc_shard_header_t &g, uint64_t max_report, arc_ve
 }
 
 // Device target for the global report (caller's device buffer, or staging).
-static int report_target(Ctx &c, arc_verify_result_t *result, uint64_t cap, arc_mismatch_t **dst, bool *host) {
+int report_target(Ctx &c, arc_verify_result_t *result, uint64_t cap, arc_mismatch_t **dst, bool *host) {
     *dst = nullptr;
     *host = false;
     if (cap == 0) return ARC_OK;
@@ -262,6 +262,15 @@ static int report_target(Ctx &c, arc_verify_result_t *result, uint64_t cap, arc_
 }
 
 int shard_compare(Ctx &c, const arc_verify_region_t &r, arc_verify_result_t *result) {
+    // the device-driven peer-memory exchange (arcv_peer.cu) when the windows are
+    // open and large enough -- uniform across ranks (same max_report, same cap)
+    if (c.peer_ready && r.max_report <= c.win_cap) return peer_compare(c, r, result);
+    if (!c.nccl_comm) {
+        set_error(c.peer_ready ? "max_report %llu exceeds the peer window capacity and no NCCL communicator"
+                               : "sharded mode needs arc_verify_peer_open or an NCCL id (max_report %llu)",
+                  (unsigned long long)r.max_report);
+        return ARC_E_UNSUPPORTED;
+    }
     int st = validate_region(r.out, r.ref, r.n, r.dtype, r.abs_tol, r.rel_tol, r.max_report, result);
     if (st) return st;
     const int p = c.nranks;

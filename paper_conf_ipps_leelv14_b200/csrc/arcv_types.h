@@ -77,6 +77,7 @@ struct Params {
     Acc *result;
     unsigned long long *done_flag;  // mapped host word: seq is stored when the call's results are final
     unsigned long long seq;
+    Acc *mirror;                    // optional device copy of the published result slots (peer exchange)
     uint32_t report_host;           // some report lives in pinned host memory (system-scope fences)
     int finalize;
     uint32_t flags;

@@ -1,0 +1,134 @@
+"""GPU parity of the sharded path over the peer-memory exchange (arcv_peer.cu).
+
+World-size 2 and 3 process groups run on ONE GPU: every rank is its own process
+with its own CUDA context, so the peer windows really are mapped through CUDA
+IPC and the exchange kernel really waits on flags stored by other processes --
+the same code that runs across the GPUs of an NVSwitch box (only the link
+differs).  torch.distributed (gloo) carries only the 64-byte window handles.
+Every rank must receive the identical global result, bit-exact against the
+unsharded CPU oracle, over several consecutive calls (both window parities).
+"""
+import os
+import socket
+import struct
+import sys
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import synth
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _bits(x):
+    return struct.unpack("<Q", struct.pack("<d", x))[0]
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _cases():
+    """(name, region factory, cuts as fractions or absolute, max_report list)."""
+    return [
+        ("C1", lambda: synth.C1(), [1e-6, 1e-5], "f32"),
+        ("C4s", lambda: synth.C4(1 << 20), [1e-6, 1e-5], "f64"),
+        ("C5s", lambda: synth.C5(1 << 16), [0.0, 0.0], "i32"),
+    ]
+
+
+def _cuts(n, world, kind):
+    if kind == "even":
+        return [r * n // world for r in range(world + 1)]
+    if kind == "ragged":
+        c = [0] + [min(n, (r + 1) * n // world + 4097 * (r + 1)) for r in range(world - 1)] + [n]
+        return c
+    if kind == "empty0":  # rank 0 holds nothing
+        return [0, 0] + [r * n // (world - 1) for r in range(1, world)]
+    raise ValueError(kind)
+
+
+def _worker(rank, world, port, q):
+    sys.path.insert(0, ROOT)
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    out = []
+    try:
+        import paper_conf_ipps_leelv14_b200 as av
+
+        torch.cuda.set_device(0)
+        assert av.init_distributed(transport="peer", max_report_cap=1 << 14) == "peer"
+        for name, mk, (at, rt), dt in _cases():
+            reg = mk()
+            for kind in ("even", "ragged", "empty0"):
+                cuts = _cuts(reg.n, world, kind)
+                a, b = cuts[rank], cuts[rank + 1]
+                o, r = reg.slice(a, b - a, device="cuda")
+                for mr in (0, 7, 100, 1 << 14):
+                    for rep in range(2):  # consecutive calls alternate the window parity
+                        g = av.compare(o, r, at, rt, mr)
+                        out.append(((name, kind, mr, rep), (g.n, g.n_mismatch, _bits(g.max_abs_err),
+                                                            _bits(g.max_rel_err), g.n_reported,
+                                                            np.array(g.report).tobytes())))
+        # a report larger than the window with no NCCL communicator: refused, not wrong
+        try:
+            av.compare(o, r, 0, 0, (1 << 14) + 1)
+            out.append((("oversize",), "accepted"))
+        except av.ArcVerifyError as e:
+            out.append((("oversize",), "refused" if e.status == av.ARC_E_UNSUPPORTED else str(e)))
+        av.finalize()
+        q.put((rank, out, None))
+    except Exception as e:  # pragma: no cover - reported to the parent
+        import traceback
+
+        q.put((rank, out, traceback.format_exc()))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.timeout(600)
+@pytest.mark.parametrize("world", [2, 3])
+def test_peer_exchange_matches_unsharded_oracle(world):
+    import oracle
+
+    oracle.build()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = {}
+    for _ in range(world):
+        rank, out, err = q.get(timeout=540)
+        assert err is None, f"rank {rank}:\n{err}"
+        res[rank] = dict(out)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    # every rank holds the identical global result
+    for r in range(1, world):
+        assert res[r] == res[0]
+    assert res[0][("oversize",)] == "refused"
+    # ... equal to the unsharded oracle
+    for name, mk, (at, rt), dt in _cases():
+        reg = mk()
+        o, r = reg.slice()
+        for mr in (0, 7, 100, 1 << 14):
+            e = oracle.compare(o.numpy(), r.numpy(), dt, at, rt, mr)
+            want = (e.n, e.n_mismatch, _bits(e.max_abs_err), _bits(e.max_rel_err), e.n_reported,
+                    np.ascontiguousarray(e.report).tobytes())
+            for kind in ("even", "ragged", "empty0"):
+                for rep in range(2):
+                    got = res[0][(name, kind, mr, rep)]
+                    assert got[:5] == want[:5], (name, kind, mr, rep, got[:5], want[:5])
+                    assert got[5] == want[5], (name, kind, mr, rep)
