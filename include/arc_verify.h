@@ -220,6 +220,11 @@ int arc_verify_get_unique_id(void *id);
 int arc_verify_set_timing(int enable);
 int arc_verify_kernel_stats(uint64_t *launches, double *total_ms, int reset);
 
+/* Number of the library's kernels launched since arc_verify_init (every kernel:
+ * compare, compact, merge / exchange, checksum); 0 before init.  Benchmarks
+ * report it as their launch count. */
+uint64_t arc_verify_launch_count(void);
+
 /*
  * arc_verify_probe_read -- DIAGNOSTIC (benchmarks only, not part of the method):
  * stream two device buffers of `bytes` each through the same bulk-copy pipeline

@@ -39,7 +39,7 @@ EXPORTED = [
     "arc_verify_version", "arc_verify_merge_plan", "arc_verify_packet_bytes",
     "arc_verify_shard_local", "arc_verify_shard_merge", "arc_verify_probe_read", "arc_verify_compare_ex",
     "arc_verify_checksum", "arc_verify_selected", "arc_verify_batch_selected", "arc_verify_format_result",
-    "arc_verify_peer_export", "arc_verify_peer_open",
+    "arc_verify_peer_export", "arc_verify_peer_open", "arc_verify_launch_count",
 ]
 
 
@@ -123,6 +123,7 @@ def _load() -> ctypes.CDLL:
                                          ctypes.c_char_p, SZ]),
         "arc_verify_peer_export": (I, [U64, P]),
         "arc_verify_peer_open": (I, [P]),
+        "arc_verify_launch_count": (U64, []),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -190,6 +191,11 @@ def arc_verify_kernel_stats(reset: bool = False) -> tuple[int, float]:
     n, ms = ctypes.c_uint64(), ctypes.c_double()
     _check(_lib.arc_verify_kernel_stats(ctypes.byref(n), ctypes.byref(ms), int(reset)), "arc_verify_kernel_stats")
     return int(n.value), float(ms.value)
+
+
+def arc_verify_launch_count() -> int:
+    """Kernels the library launched since init (every kernel it owns)."""
+    return int(_lib.arc_verify_launch_count())
 
 
 def arc_verify_version() -> int:

@@ -524,8 +524,7 @@ __device__ __forceinline__ void flush_acc(Acc *acc_base, uint32_t slot, uint32_t
 // host polls instead of a stream synchronise; system-scope fences order report
 // entries written to pinned host memory (K2, `wrote_host`) and the results
 // before that word.
-__device__ __forceinline__ void finalize_launch(const Params &p, int tid, int nthreads, int *s_last,
-                                                bool wrote_host) {
+__device__ __forceinline__ bool last_cta(const Params &p, int tid, int nthreads, int *s_last, bool wrote_host) {
     if (tid == 0) {
         if (wrote_host) __threadfence_system();
         else __threadfence();
@@ -533,7 +532,11 @@ __device__ __forceinline__ void finalize_launch(const Params &p, int tid, int nt
         *s_last = (prev - p.done_base) == (unsigned long long)(gridDim.x - 1);
     }
     if (nthreads == kConsumerThreads) consumer_bar(); else __syncthreads();
-    if (*s_last) {
+    return *s_last != 0;
+}
+
+__device__ __forceinline__ void publish(const Params &p, int tid, int nthreads) {
+    {
         __threadfence();
         for (uint32_t k = tid; k < p.n_acc; k += nthreads) {
             Acc a;
@@ -555,6 +558,11 @@ __device__ __forceinline__ void finalize_launch(const Params &p, int tid, int nt
             }
         }
     }
+}
+
+__device__ __forceinline__ void finalize_launch(const Params &p, int tid, int nthreads, int *s_last,
+                                                bool wrote_host, bool do_publish = true) {
+    if (last_cta(p, tid, nthreads, s_last, wrote_host) && do_publish) publish(p, tid, nthreads);
 }
 
 // ------------------------------------------------------------------ K1: stream
@@ -676,7 +684,13 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
         if (lane == 0) mbar_arrive(&empty_bar[s]);  // stage may be refilled now
     }
     if (cur >= 0) flush_acc(p.acc, g.acc_slot, g.dtype, acc, ctid, s_red_u, s_red_d);
-    if (p.finalize) finalize_launch(p, ctid, kConsumerThreads, &s_last, false);
+    // The last CTA publishes at once unless K2 has report entries to write: with
+    // no mismatch in any reporting region (the common "verified clean" case)
+    // the host wakes here while K2 -- then a no-op -- runs in the background.
+    if ((p.finalize || p.k2) && last_cta(p, ctid, kConsumerThreads, &s_last, false)) {
+        __threadfence();
+        if (p.finalize && (!p.k2 || *(volatile uint32_t *)p.nz_cnt == 0u)) publish(p, ctid, kConsumerThreads);
+    }
 }
 
 // --------------------------------------------------------------- K2 helpers
@@ -891,6 +905,13 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
     };
 
     const uint32_t n_nz = *(volatile uint32_t *)p.nz_cnt;
+    if (n_nz == 0) {
+        // nothing to report: K1 published; keep the grid-barrier and
+        // finished-CTA bookkeeping in step
+        if (tid == 0) atomicAdd(p.gbar, 1ull);
+        if (p.finalize) finalize_launch(p, tid, kConsumerThreads, &s_last, false, false);
+        return;
+    }
     if (n_nz <= (uint32_t)kPoolCap) {
         // ------------------------------------------------------ pool path
         // arrive on the grid-barrier counter without waiting: the host advances

@@ -263,11 +263,12 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
     p.nz_list = c.nz_list;
     p.nz_cnt = c.nz_cnt + c.parity;
     p.nz_cnt_zero = c.nz_cnt + (c.parity ^ 1);
+    p.k2 = need_compact ? 1 : 0;
     p.gbar = c.counters + 2;
     p.gbar_base = c.gbar_base;
     p.acc = c.acc + acc_lo;
     p.result = c.result_dev + acc_lo;
-    p.finalize = (finalize && !need_compact) ? 1 : 0;
+    p.finalize = finalize ? 1 : 0;  // K1 publishes unless K2 has report entries to write
     p.flags = (uint32_t)c.flags;
     p.done_flag = (c.flags & 8) ? nullptr : c.flag_dev;  // ARCV_FLAGS bit 3 (diagnostic): stream sync
     if (finalize) p.seq = ++c.seq;  // the host waits for the last finalize launch's number
@@ -285,7 +286,7 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
     if (e != cudaSuccess) return cuda_fail(e, "arcv_stream_kernel launch");
     c.launches++;
     c.ticket_base += tiles + grid;
-    if (p.finalize) c.done_base += grid;
+    if (p.finalize || p.k2) c.done_base += grid;  // K1 counts its CTAs to find its last one
     if (need_compact) {
         p.finalize = finalize ? 1 : 0;
         p.done_base = c.done_base;
@@ -641,7 +642,8 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
                 c->num_sms, c->stages, c->ctas_per_sm, occ, c->k2_grid, fa.numRegs, fa.sharedSizeBytes, smem, fa.localSizeBytes);
     }
     // counters: [0] tile tickets, [1] finished CTAs, [2] K2 grid barrier,
-    // [3] 2 x u32 active-list lengths, [4] 2 x u32 pool lengths (by parity)
+    // [3] 2 x u32 active-list lengths, [4] 2 x u32 pool lengths (by parity),
+    // [5] peer-exchange finished blocks
     e = cudaMalloc(&c->counters, 8 * sizeof(unsigned long long));
     if (e != cudaSuccess) { cudaGetLastError(); set_error("cudaMalloc counters"); return ARC_E_NOMEM; }
     CK(cudaMemsetAsync(c->counters, 0, 8 * sizeof(unsigned long long), c->stream));
@@ -651,6 +653,7 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
     CK(cudaHostGetDevicePointer(reinterpret_cast<void **>(&c->flag_dev), c->flag_host, 0));
     c->active_cnt = reinterpret_cast<uint32_t *>(c->counters + 3);
     c->nz_cnt = reinterpret_cast<uint32_t *>(c->counters + 4);
+
     e = cudaMalloc(&c->nz_list, 2 * kPoolCap * sizeof(uint64_t));
     if (e != cudaSuccess) { cudaGetLastError(); set_error("cudaMalloc pool list"); return ARC_E_NOMEM; }
     CK(cudaStreamSynchronize(c->stream));
@@ -719,6 +722,8 @@ int arc_verify_set_timing(int enable) {
     g_ctx->timing = enable != 0;
     return ARC_OK;
 }
+
+uint64_t arc_verify_launch_count(void) { return g_ctx ? g_ctx->launches : 0; }
 
 int arc_verify_kernel_stats(uint64_t *launches, double *total_ms, int reset) {
     if (!g_ctx) return ARC_E_NOINIT;

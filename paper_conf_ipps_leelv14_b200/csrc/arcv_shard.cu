@@ -215,6 +215,7 @@ static int merge_gathered(Ctx &c, const uint8_t *gathered, int p, uint64_t K, ui
     const int grid = std::max(1, std::min(c.num_sms, (int)((std::min(K, max_report) * p + 255) / 256)));
     arcv_merge_kernel<<<grid, 256, 0, c.stream>>>(gathered, p, stride, K, max_report, dst, c.merge_dev);
     CK(cudaGetLastError());
+    c.launches++;
     CK(cudaMemcpyAsync(c.hdr_host, c.merge_dev, (p + 1) * sizeof(arc_shard_header_t), cudaMemcpyDeviceToHost,
                        c.stream));
     CK(cudaStreamSynchronize(c.stream));
@@ -312,6 +313,7 @@ int shard_compare(Ctx &c, const arc_verify_region_t &r, arc_verify_result_t *res
             const int blocks = (int)std::min<uint64_t>((cnt + 255) / 256, (uint64_t)c.num_sms * 4);
             arcv_offset_kernel<<<blocks, 256, 0, c.stream>>>(dst + plan[q].prefix + K, cnt, plan[q].index_offset);
             CK(cudaGetLastError());
+            c.launches++;
         }
     }
     fill_result(g, r.max_report, result);

@@ -71,6 +71,7 @@ struct Params {
     uint64_t *nz_list;        // K1 -> K2 pool: {seg << 40 | tile, count} of nonzero tiles
     uint32_t *nz_cnt;         // this launch's pool length (may exceed kPoolCap: overflow)
     uint32_t *nz_cnt_zero;    // the other parity
+    int k2;                   // K2 follows this K1 (some segment wants a report)
     unsigned long long *gbar; // K2 grid barrier counter (monotonic)
     unsigned long long gbar_base;
     Acc *acc;
