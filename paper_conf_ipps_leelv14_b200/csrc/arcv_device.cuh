@@ -683,6 +683,9 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty_bar[s]);  // stage may be refilled now
     }
+    // K2 (programmatic dependent launch) may be scheduled from here on; it
+    // waits for this grid's completion before reading anything it wrote.
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     if (cur >= 0) flush_acc(p.acc, g.acc_slot, g.dtype, acc, ctid, s_red_u, s_red_d);
     // The last CTA publishes at once unless K2 has report entries to write: with
     // no mismatch in any reporting region (the common "verified clean" case)
@@ -858,6 +861,10 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
 
     const Seg *segs = p.segs ? p.segs : p.inline_segs;
     const int tid = threadIdx.x;
+    // launched as a programmatic dependent of K1: wait for K1's completion (and
+    // the visibility of its writes) before touching any of them
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");  // the exchange kernel, if any
     if (tid == 0) {
         mbar_init(&bar[0], 1);
         mbar_init(&bar[1], 1);

@@ -270,7 +270,8 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
     p.result = c.result_dev + acc_lo;
     p.finalize = finalize ? 1 : 0;  // K1 publishes unless K2 has report entries to write
     p.flags = (uint32_t)c.flags;
-    p.done_flag = (c.flags & 8) ? nullptr : c.flag_dev;  // ARCV_FLAGS bit 3 (diagnostic): stream sync
+    // ARCV_FLAGS bit 3 (diagnostic): stream sync; deferred (peer) calls wake on the exchange kernel
+    p.done_flag = ((c.flags & 8) || c.defer_wait) ? nullptr : c.flag_dev;
     if (finalize) p.seq = ++c.seq;  // the host waits for the last finalize launch's number
     p.mirror = finalize ? c.mirror_next : nullptr;
     for (uint32_t k = 0; k < n_segs; ++k)
@@ -291,9 +292,27 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
         p.finalize = finalize ? 1 : 0;
         p.done_base = c.done_base;
         const uint32_t grid2 = (uint32_t)c.k2_grid;
-        void *args[] = {&p};
-        e = cudaLaunchCooperativeKernel((const void *)arcv_compact_kernel, dim3(grid2), dim3(kConsumerThreads), args,
-                                        kCompactSmem, c.stream);
+        // cooperative (the group path has a grid barrier) and, unless disabled,
+        // a programmatic dependent of K1: its launch overlaps K1's tail
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(grid2);
+        cfg.blockDim = dim3(kConsumerThreads);
+        cfg.dynamicSmemBytes = kCompactSmem;
+        cfg.stream = c.stream;
+        cudaLaunchAttribute at[2];
+        at[0].id = cudaLaunchAttributeCooperative;
+        at[0].val.cooperative = 1;
+        at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        at[1].val.programmaticStreamSerializationAllowed = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = c.pdl ? 2 : 1;
+        e = cudaLaunchKernelEx(&cfg, arcv_compact_kernel, p);
+        if (e != cudaSuccess && c.pdl) {  // PDL refused with a cooperative launch: plain cooperative
+            cudaGetLastError();
+            c.pdl = false;
+            cfg.numAttrs = 1;
+            e = cudaLaunchKernelEx(&cfg, arcv_compact_kernel, p);
+        }
         if (e != cudaSuccess) return cuda_fail(e, "arcv_compact_kernel cooperative launch");
         c.launches++;
         c.gbar_base += grid2;
@@ -618,6 +637,7 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
         CK(cudaEventCreate(&c->ev[i][1]));
     }
     c->flags = env_int("ARCV_FLAGS", 0);
+    c->pdl = env_int("ARCV_PDL", 1) != 0;
     c->stages = env_int("ARCV_STAGES", 3);
     if (c->stages != 2 && c->stages != 3 && c->stages != 4 && c->stages != 6) c->stages = 3;
     const size_t smem = (size_t)c->stages * kStageBytes;

@@ -64,6 +64,7 @@ struct PeerParams {
     uint64_t n_local, max_report, cap;
     const Acc *mirror;              // local summary (written by the local compare)
     arc_mismatch_t *dst;            // global report target (device or pinned alias), or nullptr
+    int dst_host;                   // dst is mapped host memory (system-scope fences)
     arc_shard_header_t *out;        // mapped host: [0] global header, [1].n = status (1 = timeout)
     unsigned long long *done;       // monotonic finished-block counter
     unsigned long long done_base;
@@ -96,6 +97,7 @@ __global__ void __launch_bounds__(256) arcv_peer_kernel(const __grid_constant__ 
     __shared__ int s_ok, s_last;
     const int tid = threadIdx.x;
     uint8_t *own = q.win[q.rank];
+    asm volatile("griddepcontrol.wait;" ::: "memory");  // the local compare has completed
 
     // 1. publish (one thread of the grid)
     if (blockIdx.x == 0 && tid == 0) {
@@ -164,7 +166,8 @@ __global__ void __launch_bounds__(256) arcv_peer_kernel(const __grid_constant__ 
     __syncthreads();
     if (tid == 0) {
         if (!ok) q.out[1].n = 1;  // status: timed out
-        __threadfence_system();
+        if (q.dst_host || !ok) __threadfence_system();
+        else __threadfence();
         const unsigned long long prev = atomicAdd(q.done, 1ull);
         s_last = (prev - q.done_base) == (unsigned long long)(gridDim.x - 1);
     }
@@ -240,15 +243,25 @@ int peer_compare(Ctx &c, const arc_verify_region_t &r, arc_verify_result_t *resu
     q.cap = c.win_cap;
     q.mirror = c.mirror;
     q.dst = dst;
+    q.dst_host = 0;
     q.out = c.peer_out_dev;
     q.done = c.counters + 5;
     q.done_base = c.peer_done_base;
     q.done_flag = c.flag_dev;
     q.seq = ++c.seq;
+    // a few blocks: the merge moves <= max_report x 24 B, mostly a handful
     const uint64_t work = std::min<uint64_t>(r.max_report, 1ull << 40);
-    const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)c.num_sms, (work + 255) / 256));
-    arcv_peer_kernel<<<grid, 256, 0, c.stream>>>(q);
-    CK(cudaGetLastError());
+    const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(32, (work + 2047) / 2048));
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(256);
+    cfg.stream = c.stream;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = c.pdl ? 1 : 0;
+    CK(cudaLaunchKernelEx(&cfg, arcv_peer_kernel, q));
     c.launches++;
     c.peer_done_base += (unsigned long long)grid;
     st = wait_results(c);
