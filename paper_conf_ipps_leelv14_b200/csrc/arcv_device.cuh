@@ -735,6 +735,8 @@ __device__ __noinline__ void compact_tile(const Seg &g, const StageInfo &si, con
         packed |= (uint64_t)__popcll(mask & (kGroup << (k * EPV))) << (16 * k);
     uint64_t total;
     const uint64_t ex = block_excl_scan(packed, s_w, &total);
+    arc_mismatch_t *const rep = (excl & kDirectBit) ? g.report_alias : g.report;
+    excl &= ~kDirectBit;
     uint64_t m = mask;
     while (m) {
         const int b = __ffsll((long long)m) - 1;
@@ -748,7 +750,7 @@ __device__ __noinline__ void compact_tile(const Seg &g, const StageInfo &si, con
             const uint32_t te = (uint32_t)((k * kConsumerThreads + tid) * EPV + j);  // tile element
             const T xo = *reinterpret_cast<const T *>(so + si.off_o + te * sizeof(T));  // from the stage
             const T xr = *reinterpret_cast<const T *>(sr + si.off_r + te * sizeof(T));
-            arc_mismatch_t *dst = g.report + gi;
+            arc_mismatch_t *dst = rep + gi;
             dst->index = g.index_base + si.elem_begin + te;
             dst->out_bits = raw_bits<T>(xo);
             dst->ref_bits = raw_bits<T>(xr);
@@ -856,6 +858,7 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
     __shared__ uint64_t s_loc_pre[kPoolLocal];
     __shared__ uint32_t s_n;
     __shared__ int s_last;
+    __shared__ int s_wrote;  // this CTA wrote report entries to pinned host memory
     uint64_t *s_pkey = reinterpret_cast<uint64_t *>(smem + 2 * kStageBytes);
     uint32_t *s_pcnt = reinterpret_cast<uint32_t *>(s_pkey + kPoolCap);
 
@@ -866,6 +869,7 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
     asm volatile("griddepcontrol.wait;" ::: "memory");
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");  // the exchange kernel, if any
     if (tid == 0) {
+        s_wrote = 0;
         mbar_init(&bar[0], 1);
         mbar_init(&bar[1], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -950,8 +954,13 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
             if (tid == 0) {
                 p.tile_cnt[g.slot_begin + lt] = 0u;  // clean for the next call
                 if (base + pre_tot < g.max_report && s_n < (uint32_t)kPoolLocal) {
+                    // a sparse region with a pinned host report: written over PCIe
+                    // directly (the host then skips its D2H copy; same rule there)
+                    const bool direct =
+                        g.report_alias && !(g.flags & kSegBaseFromAcc) && seg_tot <= kDirectDyn;
                     s_loc_key[s_n] = key;
-                    s_loc_pre[s_n] = base + pre_tot;
+                    s_loc_pre[s_n] = (base + pre_tot) | (direct ? kDirectBit : 0ull);
+                    s_wrote |= direct;
                     s_n = s_n + 1;
                 }
             }
@@ -1022,7 +1031,7 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
         process(mine, [&](uint32_t j) { return __ldcg(p.active + 2 * (blockIdx.x + j * gridDim.x)); },
                 [&](uint32_t j) { return __ldcg(p.active + 2 * (blockIdx.x + j * gridDim.x) + 1); });
     }
-    if (p.finalize) finalize_launch(p, tid, kConsumerThreads, &s_last, p.report_host != 0);
+    if (p.finalize) finalize_launch(p, tid, kConsumerThreads, &s_last, p.report_host != 0 || s_wrote != 0);
 }
 
 }  // namespace arcv

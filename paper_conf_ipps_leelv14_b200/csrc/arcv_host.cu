@@ -116,8 +116,9 @@ PtrKind classify(const void *p, int device) {
 
 constexpr int kCompactSmem = 2 * kStageBytes + kPoolCap * (8 + 4);
 
-// Pinned host reports up to this many entries are written by the kernel over
-// PCIe; larger ones are staged in HBM and copied with one bulk D2H.
+// Pinned host reports with a capacity up to Ctx::direct_max entries are
+// written by the kernel over PCIe; larger ones are staged in HBM and copied
+// with one bulk D2H (ARCV_DIRECT_MAX overrides the default).
 constexpr uint64_t kDirectReportMax = 1 << 16;
 
 // Device alias of page-locked host memory (cudaMallocHost / cudaHostRegister /
@@ -445,6 +446,7 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
     struct Plan {
         bool out_dev, ref_dev, stream;
         arc_mismatch_t *dreport;  // device target
+        arc_mismatch_t *alias;    // device alias of a pinned host report (sparse: written directly)
         bool host_report;
         uint64_t stage_off;
         uint64_t tiles, slot_base;
@@ -475,17 +477,19 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
         const uint64_t cap = std::min<uint64_t>(r.max_report, r.n);
         pl.host_report = false;
         pl.dreport = nullptr;
+        pl.alias = nullptr;
         if (cap > 0) {
             if (dev_reports) {
                 pl.dreport = dev_reports[k];
             } else if (classify(results[k].report, c.device) == PK_DEVICE) {
                 pl.dreport = results[k].report;
-            } else if (void *alias = cap <= kDirectReportMax ? pinned_device_alias(results[k].report) : nullptr) {
+            } else if (void *alias = cap <= c.direct_max ? pinned_device_alias(results[k].report) : nullptr) {
                 pl.dreport = static_cast<arc_mismatch_t *>(alias);  // small pinned report: written over PCIe by K2
             } else {
                 pl.host_report = true;
                 pl.stage_off = stage_entries;
                 stage_entries += cap;
+                if (!pl.stream) pl.alias = static_cast<arc_mismatch_t *>(pinned_device_alias(results[k].report));
             }
         }
     }
@@ -509,6 +513,7 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
         slot_of[k] = next_slot;
         segs.push_back(make_seg(r.out, r.ref, r.n, (uint32_t)r.dtype, r.abs_tol, r.rel_tol, r.max_report,
                                 plan[k].dreport, plan[k].slot_base, 0, next_slot, 0, r.check));
+        segs.back().report_alias = plan[k].alias;
         next_slot++;
     }
     const uint32_t n_dev_slots = next_slot;
@@ -555,6 +560,7 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
         bool any = false;
         for (size_t k = 0; k < R; ++k) {
             if (!plan[k].host_report || results[k].n_reported == 0) continue;
+            if (plan[k].alias && results[k].n_mismatch <= kDirectDyn) continue;  // K2 wrote it directly
             CK(cudaMemcpyAsync(results[k].report, plan[k].dreport, results[k].n_reported * sizeof(arc_mismatch_t),
                                cudaMemcpyDeviceToHost, c.stream));
             any = true;
@@ -638,6 +644,10 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
     }
     c->flags = env_int("ARCV_FLAGS", 0);
     c->pdl = env_int("ARCV_PDL", 1) != 0;
+    {
+        const char *v = getenv("ARCV_DIRECT_MAX");
+        c->direct_max = (v && *v) ? strtoull(v, nullptr, 0) : kDirectReportMax;
+    }
     c->stages = env_int("ARCV_STAGES", 3);
     if (c->stages != 2 && c->stages != 3 && c->stages != 4 && c->stages != 6) c->stages = 3;
     const size_t smem = (size_t)c->stages * kStageBytes;

@@ -22,6 +22,7 @@ struct Ctx {
     bool sharded = false;  // collective path (NCCL communicator), nranks >= 1
     int num_sms = 0, ctas_per_sm = 1, stages = 3, flags = 0;
     int k2_grid = 0;  // K2 (cooperative) grid: SMs x co-resident CTAs (<= 2)
+    uint64_t direct_max = 0;  // pinned host reports up to this capacity: written by the kernel
     bool pdl = true;  // launch K2 / the exchange kernel as programmatic dependents (ARCV_PDL=0: off)
     cudaStream_t stream = nullptr;
     bool own_stream = false;

@@ -18,6 +18,8 @@ constexpr int kMaxInlineSegs = 8;
 constexpr int kGroupTiles = 256;                    // tiles per group counter
 constexpr int kPoolCap = 2048;                      // K2 pool path: max listed nonzero tiles
 constexpr int kPoolLocal = 64;                      // per-CTA share of the pool (grid >= 32)
+constexpr uint64_t kDirectDyn = 4096;               // sparse reports: K2 writes a pinned host report directly
+constexpr uint64_t kDirectBit = 1ull << 63;         // K2 tile prefix flag: entries go to report_alias
 static_assert(kVecPerThread == 4, "packed-scan layout assumes 4 vectors per thread");
 static_assert(kGroupTiles == kConsumerThreads, "K2 scans one group per block pass");
 
@@ -37,6 +39,9 @@ struct Seg {
     double abs_tol, rel_tol;
     uint64_t max_report;    // report capacity / truncation for the region (0 = count only)
     arc_mismatch_t *report; // device pointer, entries [0, max_report)
+    arc_mismatch_t *report_alias;  // device alias of the caller's pinned host report, or nullptr:
+                                   // used instead of `report` when the region has <= kDirectDyn
+                                   // mismatches (then the host skips the D2H copy)
     uint32_t acc_slot;
     uint32_t dtype;
     uint32_t flags;

@@ -436,6 +436,31 @@ def test_pinned_report(av, orc, mr):
     assert_same(g, o, f"pinned mr={mr}")
 
 
+@pytest.mark.parametrize("n_mis", [0, 1, 4095, 4096, 4097, 20000])
+def test_pinned_report_sparse_direct(av, orc, n_mis):
+    """A large pinned host report (capacity > 2^16) with <= 4096 mismatches is written by K2
+    over PCIe (no D2H copy); with more it goes through HBM staging.  Both sides of the 4096
+    boundary, a stale buffer (pre-filled with garbage) and a batch with two such regions."""
+    n = 1 << 22
+    gen = torch.Generator().manual_seed(n_mis + 7)
+    ref = torch.randint(-(1 << 30), 1 << 30, (n,), generator=gen, dtype=torch.int32)
+    out = ref.clone()
+    idx = torch.randperm(n, generator=gen)[:n_mis]
+    out[idx] ^= 5
+    mr = 1 << 20
+    rep = torch.empty(24 * mr, dtype=torch.uint8, pin_memory=True).numpy().view(av.REPORT_DTYPE)
+    rep.view(np.uint8)[:] = 0xA5
+    o = orc.compare(out.numpy(), ref.numpy(), "i32", 0, 0, mr)
+    for _ in range(2):
+        g = av.compare(out.cuda(), ref.cuda(), 0, 0, mr, report=rep)
+        assert_same(g, o, f"sparse direct n_mis={n_mis}")
+    if n_mis in (1, 4097):
+        res = av.batch([(out.cuda(), ref.cuda(), 0, 0, mr), (ref.cuda(), out.cuda(), 0, 0, mr)])
+        o2 = orc.compare(ref.numpy(), out.numpy(), "i32", 0, 0, mr)
+        assert_same(res[0], o, "batch 0")
+        assert_same(res[1], o2, "batch 1")
+
+
 @pytest.mark.parametrize("n", [1, 15, 16, 17, 16384 * 3 + 5, (1 << 22) + 3])
 def test_u8_simd_path(av, orc, n):
     gen = torch.Generator().manual_seed(n)

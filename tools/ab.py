@@ -170,6 +170,22 @@ add("C4", c4)
 add("C5", c5)
 
 print(f"libs: {libs}; rounds {ROUNDS} x {STEPS} steps", flush=True)
+if not ONLY or "probe" in ONLY.split(","):
+    for nb in (1 << 28, 1 << 32):
+        a_ = torch.empty(nb, dtype=torch.uint8, device="cuda")
+        b_ = torch.empty(nb, dtype=torch.uint8, device="cuda")
+        res_ = [[] for _ in L]
+        for rd in range(ROUNDS):
+            for k, lib in enumerate(L):
+                g = ctypes.c_double()
+                assert lib.arc_verify_probe_read(ctypes.c_void_p(a_.data_ptr()), ctypes.c_void_p(b_.data_ptr()),
+                                                 ctypes.c_uint64(nb), 10, ctypes.byref(g)) == 0
+                res_[k].append(g.value)
+        print(f"probe {nb >> 20:6d} MiB/array " + " ".join(
+            f"| {os.path.basename(libs[k])[:18]:18s} {statistics.median(res_[k]):8.1f} GB/s" for k in range(len(L))),
+            flush=True)
+        del a_, b_
+        torch.cuda.empty_cache()
 for name, make in W.items():
     mk, nbytes = make()
     calls = [mk(k) for k in range(len(L))]
