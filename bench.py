@@ -40,7 +40,8 @@ def parse():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--n", type=int, default=N_C4, help="elements per array (default: C4's 2^29)")
+    ap.add_argument("--n", "--n-elements", dest="n", type=int, default=N_C4,
+                    help="elements per array (default: C4's 2^29); --n-elements under torchrun")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -193,15 +194,24 @@ def main():
     import synth
 
     assert world == args.gpus, f"--gpus {args.gpus} but WORLD_SIZE {world}"
-    torch.cuda.set_device(local_rank)
+    # ARCV_BENCH_ONE_GPU=1 (diagnostic, tests only): every rank on cuda:0, gloo for
+    # the host-side collectives, peer windows between the processes -- exercises
+    # the N > 1 code path on a one-GPU box (its numbers mean nothing)
+    one_gpu = os.environ.get("ARCV_BENCH_ONE_GPU") == "1"
+    dev = 0 if one_gpu else local_rank
+    torch.cuda.set_device(dev)
     exchange = None
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if one_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
         # the device-driven peer-memory exchange (CUDA IPC windows over NVLink);
         # NCCL only as the fallback when the windows cannot be mapped
-        exchange = av.init_distributed(transport="auto", max_report_cap=1 << 20)
+        exchange = av.init_distributed(transport="peer" if one_gpu else "auto", max_report_cap=1 << 20)
     else:
-        av.init(local_rank)
+        av.init(dev)
+    red_dev = "cpu" if one_gpu else "cuda"
 
     n = args.n
     lo, hi = rank * n // world, (rank + 1) * n // world
@@ -229,7 +239,7 @@ def main():
     launches0 = av.arc_verify_launch_count()
     stream = torch.cuda.current_stream()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    sampler = ClockSampler(local_rank) if not args.profile else None
+    sampler = ClockSampler(dev) if not args.profile else None
     barrier()
     if sampler:
         sampler.__enter__()
@@ -244,7 +254,7 @@ def main():
     gpu_launches = av.arc_verify_launch_count() - launches0
     launches, kern_ms = av.arc_verify_kernel_stats(reset=True)
     av.arc_verify_set_timing(False)
-    t = torch.tensor([ms, kern_ms / max(launches, 1)], dtype=torch.float64, device="cuda")
+    t = torch.tensor([ms, kern_ms / max(launches, 1)], dtype=torch.float64, device=red_dev)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     ms_max, kern_avg_ms = float(t[0]), float(t[1])
@@ -280,7 +290,7 @@ def main():
             rh = step_h()
         t1.record(stream)
         torch.cuda.synchronize()
-        te = torch.tensor([t0.elapsed_time(t1)], dtype=torch.float64, device="cuda")
+        te = torch.tensor([t0.elapsed_time(t1)], dtype=torch.float64, device=red_dev)
         if world > 1:
             dist.all_reduce(te, op=dist.ReduceOp.MAX)
         e2e_ms = float(te[0])
@@ -300,7 +310,7 @@ def main():
             rr = step_r()
         t1.record(stream)
         torch.cuda.synchronize()
-        te = torch.tensor([t0.elapsed_time(t1)], dtype=torch.float64, device="cuda")
+        te = torch.tensor([t0.elapsed_time(t1)], dtype=torch.float64, device=red_dev)
         if world > 1:
             dist.all_reduce(te, op=dist.ReduceOp.MAX)
         parity = parity and rr.n_mismatch == res.n_mismatch

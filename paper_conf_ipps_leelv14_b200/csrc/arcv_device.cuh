@@ -764,42 +764,62 @@ __device__ __noinline__ void compact_tile(const Seg &g, const StageInfo &si, con
 // small code matters here because every CTA executes it cold, once.
 // The decision is the same rule K1 applies (its fast path only ever proves
 // matches), so the in-tile ranks agree with K1's counts.
+// Scalars by value: references to SegHot / StageInfo would put them in local
+// memory (the function is not inlined) and reload them every iteration.
 template <typename T>
-__device__ __noinline__ uint64_t mask_tile(const uint8_t *so, const uint8_t *sr, const StageInfo &si, int tid,
-                                           const SegHot &g) {
+__device__ __noinline__ uint64_t mask_tile(const uint8_t *so, const uint8_t *sr, uint32_t count, uint32_t off_o,
+                                           uint32_t off_r, int tid, double abs_tol, double rel_tol, uint32_t cflags,
+                                           double minv, double lo, double hi) {
     constexpr int EPV = 16 / sizeof(T);
     uint64_t mask = 0;
+    if constexpr (!std::is_floating_point<T>::value) {
+        if (cflags == 0) {  // integers: plain equality
+#pragma unroll 4
+            for (int b = 0; b < kVecPerThread * EPV; ++b) {
+                const uint32_t e = (uint32_t)(((b / EPV) * kConsumerThreads + tid) * EPV + (b % EPV));
+                if (e >= count) continue;
+                const T xo = *reinterpret_cast<const T *>(so + off_o + e * sizeof(T));
+                const T yr = *reinterpret_cast<const T *>(sr + off_r + e * sizeof(T));
+                mask |= (uint64_t)(xo != yr) << b;
+            }
+            return mask;
+        }
+    }
 #pragma unroll 1
     for (int b = 0; b < kVecPerThread * EPV; ++b) {
         const uint32_t e = (uint32_t)(((b / EPV) * kConsumerThreads + tid) * EPV + (b % EPV));
-        if (e >= si.count) continue;
-        const T xo = *reinterpret_cast<const T *>(so + si.off_o + e * sizeof(T));
-        const T yr = *reinterpret_cast<const T *>(sr + si.off_r + e * sizeof(T));
+        if (e >= count) continue;
+        const T xo = *reinterpret_cast<const T *>(so + off_o + e * sizeof(T));
+        const T yr = *reinterpret_cast<const T *>(sr + off_r + e * sizeof(T));
         const double x = (double)xo, y = (double)yr;
-        if ((g.cflags & ARC_CHECK_MIN_VALUE) && fabs(y) <= g.minv) continue;
+        if ((cflags & ARC_CHECK_MIN_VALUE) && fabs(y) <= minv) continue;
         bool mis;
         if constexpr (std::is_floating_point<T>::value) {
             const double d = fabs(x - y);
-            const double t = __dadd_rn(g.abs_tol, __dmul_rn(g.rel_tol, fabs(y)));
+            const double t = __dadd_rn(abs_tol, __dmul_rn(rel_tol, fabs(y)));
             mis = !((x == y) | ((x != x) & (y != y)) | ((fabs(y) < CUDART_INF) & (d <= t)));
         } else {
             mis = xo != yr;
         }
-        if (mis && (g.cflags & ARC_CHECK_VALUE_BOUNDS) && g.lo <= x && x <= g.hi) mis = false;
+        if (mis && (cflags & ARC_CHECK_VALUE_BOUNDS) && lo <= x && x <= hi) mis = false;
         mask |= (uint64_t)mis << b;
     }
     return mask;
 }
 
+template <typename G>
 __device__ __forceinline__ uint64_t mask_any(const uint8_t *so, const uint8_t *sr, const StageInfo &si, int tid,
-                                             const SegHot &g) {
+                                             const G &g) {
+#define ARCV_MASK(T) mask_tile<T>(so, sr, si.count, si.off_o, si.off_r, tid, g.abs_tol, g.rel_tol, g.cflags, \
+                                  g.minv, g.lo, g.hi)
     switch (g.dtype) {
-        case ARC_F32: return mask_tile<float>(so, sr, si, tid, g);
-        case ARC_F64: return mask_tile<double>(so, sr, si, tid, g);
-        case ARC_I32: return mask_tile<int32_t>(so, sr, si, tid, g);
-        case ARC_I64: return mask_tile<int64_t>(so, sr, si, tid, g);
-        default: return mask_tile<uint8_t>(so, sr, si, tid, g);
+        case ARC_F32: return ARCV_MASK(float);
+        case ARC_F64: return ARCV_MASK(double);
+        case ARC_I32: return ARCV_MASK(int32_t);
+        case ARC_I64: return ARCV_MASK(int64_t);
+        default: return ARCV_MASK(uint8_t);
     }
+#undef ARCV_MASK
 }
 
 // ---------------------------------------------------------------- K2: compact
@@ -932,9 +952,17 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
             s_pkey[i] = __ldcg(p.nz_list + 2 * i);
             s_pcnt[i] = (uint32_t)__ldcg(p.nz_list + 2 * i + 1);
         }
-        if (tid == 0) s_n = 0;
         __syncthreads();
-        for (uint32_t k = blockIdx.x; k < n_nz; k += gridDim.x) {
+        // This CTA's pool entries k = blockIdx.x + j * gridDim.x.  Their tile
+        // re-reads are issued first (two stages), so the copies' latency overlaps
+        // the prefix scans; an entry whose prefix is past max_report just drops
+        // its (completed) copy.
+        const uint32_t n_own = n_nz > blockIdx.x ? (n_nz - blockIdx.x + gridDim.x - 1) / gridDim.x : 0u;
+        if (tid == 0)
+            for (uint32_t j = 0; j < n_own && j < 2; ++j) issue(s_pkey[blockIdx.x + j * gridDim.x], (int)j);
+        for (uint32_t j = 0; j < n_own; ++j) {
+            const int st = (int)(j & 1);
+            const uint32_t k = blockIdx.x + j * gridDim.x;
             const uint64_t key = s_pkey[k];
             const uint64_t seg = key >> 40, lt = key & kLtMask;
             uint64_t pre = 0, segtot = 0;
@@ -951,23 +979,26 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
             const Seg &g = segs[seg];
             uint64_t base = 0;
             if (g.flags & kSegBaseFromAcc) base = __ldcg(&p.acc[g.acc_slot].count) - seg_tot;
-            if (tid == 0) {
-                p.tile_cnt[g.slot_begin + lt] = 0u;  // clean for the next call
-                if (base + pre_tot < g.max_report && s_n < (uint32_t)kPoolLocal) {
-                    // a sparse region with a pinned host report: written over PCIe
-                    // directly (the host then skips its D2H copy; same rule there)
-                    const bool direct =
-                        g.report_alias && !(g.flags & kSegBaseFromAcc) && seg_tot <= kDirectDyn;
-                    s_loc_key[s_n] = key;
-                    s_loc_pre[s_n] = (base + pre_tot) | (direct ? kDirectBit : 0ull);
-                    s_wrote |= direct;
-                    s_n = s_n + 1;
-                }
+            const uint64_t excl = base + pre_tot;
+            if (tid == 0) p.tile_cnt[g.slot_begin + lt] = 0u;  // clean for the next call
+            mbar_wait(&bar[st], phase[st]);
+            phase[st] ^= 1u;
+            if (excl < g.max_report) {  // uniform
+                // a sparse region with a pinned host report: written over PCIe
+                // directly (the host then skips its D2H copy; same rule there)
+                const bool direct = g.report_alias && !(g.flags & kSegBaseFromAcc) && seg_tot <= kDirectDyn;
+                if (direct && tid == 0) s_wrote = 1;
+                StageInfo si;
+                uintptr_t ao, ar;
+                uint32_t nbo, nbr;
+                plan_tile(g, lt, si, ao, nbo, ar, nbr);
+                const uint8_t *so = smem + (size_t)st * kStageBytes;
+                const uint64_t mask = mask_any(so, so + kStageArrayBytes, si, tid, g);
+                compact_any(g, si, so, so + kStageArrayBytes, mask, excl | (direct ? kDirectBit : 0ull), s_w);
             }
+            __syncthreads();  // stage `st` and s_w are reused
+            if (tid == 0 && j + 2 < n_own) issue(s_pkey[k + 2 * gridDim.x], st);
         }
-        __syncthreads();
-        const uint32_t n_loc = s_n;
-        process(n_loc, [&](uint32_t j) { return s_loc_key[j]; }, [&](uint32_t j) { return s_loc_pre[j]; });
     } else {
         // ------------------------------------------------------ group path
         for (uint32_t sgi = 0; sgi < p.n_segs; ++sgi) {

@@ -9,7 +9,7 @@ set -u
 TAG=${1:-prof}
 OUT=gpurun_out
 NCU=/usr/local/cuda/bin/ncu
-$NCU --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none -c 40 --csv \
+$NCU --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none -k regex:arcv_ -c 40 --csv \
   --log-file $OUT/${TAG}_launches_c4.csv python bench.py --profile --steps 4 --warmup 3 > $OUT/${TAG}_launches_run.log 2>&1
 echo "launches rc=$?"
 $NCU --set full --clock-control none --import-source on -k regex:arcv_stream_kernel -s 3 -c 1 \
