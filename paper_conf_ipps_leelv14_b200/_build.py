@@ -53,12 +53,16 @@ def _stale() -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not _stale():
+def build(force: bool = False, verbose: bool = False, out: str | None = None, defines: tuple = ()) -> str:
+    """Build the library (in-tree by default).  `out` + `defines` build an A/B
+    variant elsewhere (e.g. scratch/var.so with -DARCV_FENCE_SC=1)."""
+    target = out or LIB
+    if out is None and not force and not _stale():
         return LIB
     nvcc = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
-    tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [nvcc, *NVCC_FLAGS, "-I", INCLUDE, "-I", CSRC, "-I", _nccl_include(), "-o", tmp, *sources(), "-ldl"]
+    tmp = target + f".tmp{os.getpid()}"
+    cmd = [nvcc, *NVCC_FLAGS, *defines, "-I", INCLUDE, "-I", CSRC, "-I", _nccl_include(), "-o", tmp, *sources(),
+           "-ldl"]
     res = subprocess.run(cmd, capture_output=True, text=True)
     log = os.path.join(HERE, "build.log")
     with open(log, "w") as f:
@@ -68,9 +72,14 @@ def build(force: bool = False, verbose: bool = False) -> str:
         raise RuntimeError(f"nvcc failed (see {log})")
     if verbose:
         sys.stderr.write(res.stderr)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, target)
+    return target
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose=True))
+    # python _build.py [--force] | python _build.py --variant OUT.so -DNAME=VALUE ...
+    if "--variant" in sys.argv:
+        i = sys.argv.index("--variant")
+        print(build(out=os.path.abspath(sys.argv[i + 1]), defines=tuple(a for a in sys.argv[i + 2:] if a.startswith("-D"))))
+    else:
+        print(build(force="--force" in sys.argv, verbose=True))

@@ -82,6 +82,42 @@ __device__ __forceinline__ void consumer_bar() {
     asm volatile("bar.sync 1, %0;" ::"n"(kConsumerThreads) : "memory");
 }
 
+// Release/acquire fences for the message-passing patterns of this file (last
+// CTA publishes; report entries before a completion word; grid barrier).  None
+// of them needs the single total order of fence.sc (what __threadfence() and
+// __threadfence_system() emit: MEMBAR.SC.GPU / MEMBAR.SC.SYS); fence.acq_rel
+// (MEMBAR.ALL.*) gives the same release and acquire patterns, cheaper.
+// -DARCV_FENCE_SC=1 restores the SC fences (A/B builds).
+__device__ __forceinline__ void fence_gpu() {
+#if defined(ARCV_FENCE_SC) && ARCV_FENCE_SC
+    __threadfence();
+#else
+    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+#endif
+}
+__device__ __forceinline__ void fence_sys() {
+#if defined(ARCV_FENCE_SC) && ARCV_FENCE_SC
+    __threadfence_system();
+#else
+    asm volatile("fence.acq_rel.sys;" ::: "memory");
+#endif
+}
+
+// Diagnostic phase trace (A/B builds only, -DARCV_TRACE=1): %globaltimer stamps
+// per CTA, read by arc_verify_debug_trace.  Compiled out otherwise.
+#if defined(ARCV_TRACE) && ARCV_TRACE
+constexpr int kTraceCtas = 1024, kTracePts = 12;
+__device__ unsigned long long g_trace[2][kTraceCtas][kTracePts];  // [kernel][cta][point]
+#define ARCV_STAMP(k, pt)                                                                      \
+    do {                                                                                       \
+        unsigned long long t_;                                                                 \
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));                               \
+        if (blockIdx.x < (unsigned)kTraceCtas) g_trace[k][blockIdx.x][pt] = t_;                \
+    } while (0)
+#else
+#define ARCV_STAMP(k, pt) do {} while (0)
+#endif
+
 __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
@@ -524,12 +560,13 @@ __device__ __forceinline__ void flush_acc(Acc *acc_base, uint32_t slot, uint32_t
 // host polls instead of a stream synchronise; system-scope fences order report
 // entries written to pinned host memory (K2, `wrote_host`) and the results
 // before that word.
-__device__ __forceinline__ bool last_cta(const Params &p, int tid, int nthreads, int *s_last, bool wrote_host) {
+__device__ __forceinline__ bool last_cta(const Params &p, int tid, int nthreads, int *s_last, bool wrote_host,
+                                         unsigned long long base) {
     if (tid == 0) {
-        if (wrote_host) __threadfence_system();
-        else __threadfence();
+        if (wrote_host) fence_sys();
+        else fence_gpu();
         const unsigned long long prev = atomicAdd(p.done, 1ull);
-        *s_last = (prev - p.done_base) == (unsigned long long)(gridDim.x - 1);
+        *s_last = (prev - base) == (unsigned long long)(gridDim.x - 1);
     }
     if (nthreads == kConsumerThreads) consumer_bar(); else __syncthreads();
     return *s_last != 0;
@@ -537,7 +574,7 @@ __device__ __forceinline__ bool last_cta(const Params &p, int tid, int nthreads,
 
 __device__ __forceinline__ void publish(const Params &p, int tid, int nthreads) {
     {
-        __threadfence();
+        fence_gpu();
         for (uint32_t k = tid; k < p.n_acc; k += nthreads) {
             Acc a;
             a.count = __ldcg(&p.acc[k].count);
@@ -553,7 +590,7 @@ __device__ __forceinline__ void publish(const Params &p, int tid, int nthreads) 
         if (p.done_flag) {
             if (nthreads == kConsumerThreads) consumer_bar(); else __syncthreads();
             if (tid == 0) {
-                __threadfence_system();
+                fence_sys();
                 *(volatile unsigned long long *)p.done_flag = p.seq;
             }
         }
@@ -561,146 +598,16 @@ __device__ __forceinline__ void publish(const Params &p, int tid, int nthreads) 
 }
 
 __device__ __forceinline__ void finalize_launch(const Params &p, int tid, int nthreads, int *s_last,
-                                                bool wrote_host, bool do_publish = true) {
-    if (last_cta(p, tid, nthreads, s_last, wrote_host) && do_publish) publish(p, tid, nthreads);
-}
-
-// ------------------------------------------------------------------ K1: stream
-template <int S, int MINB>
-__global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __grid_constant__ Params p) {
-    extern __shared__ __align__(128) uint8_t smem[];
-    __shared__ __align__(8) uint64_t full_bar[S];
-    __shared__ __align__(8) uint64_t empty_bar[S];
-    __shared__ StageInfo info[S];
-    __shared__ uint64_t s_red_u[kConsumerWarps][2];
-    __shared__ double s_red_d[kConsumerWarps][2];
-    __shared__ int s_last;
-    __shared__ uint32_t s_tile[S];
-
-    const Seg *segs = p.segs ? p.segs : p.inline_segs;
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-
-    if (threadIdx.x == 0) {
-        for (int s = 0; s < S; ++s) {
-            s_tile[s] = 0u;
-            mbar_init(&full_bar[s], 1);
-            mbar_init(&empty_bar[s], kConsumerWarps);
-        }
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncthreads();
-
-    // ------------------------------------------------------------ producer
-    if (warp == 0) {
-        if (lane == 0) {
-            const uint64_t policy = evict_first_policy();
-            for (uint32_t i = 0;; ++i) {
-                const int s = i % S;
-                if (i >= (uint32_t)S) mbar_wait(&empty_bar[s], ((i / S) - 1) & 1);
-                const uint64_t t = atomicAdd(p.ticket, 1ull) - p.ticket_base;
-                if (t >= p.total_tiles) {
-                    info[s].tile = ~0ull;
-                    mbar_arrive(&full_bar[s]);
-                    break;
-                }
-                const uint32_t sg = find_seg(segs, p.n_segs, t);
-                const Seg &g = segs[sg];
-                StageInfo &si = info[s];
-                uintptr_t ao, ar;
-                uint32_t nbo, nbr;
-                plan_tile(g, t - g.tile_begin, si, ao, nbo, ar, nbr);
-                si.tile = t;
-                si.seg = sg;
-                uint8_t *dst = smem + (size_t)s * kStageBytes;
-                mbar_arrive_expect_tx(&full_bar[s], nbo + nbr);
-                bulk_g2s(dst, reinterpret_cast<const void *>(ao), nbo, &full_bar[s], policy);
-                bulk_g2s(dst + kStageArrayBytes, reinterpret_cast<const void *>(ar), nbr, &full_bar[s], policy);
-            }
-        }
-        return;
-    }
-
-    // ------------------------------------------------------------ consumers
-    const int ctid = threadIdx.x - 32;
-    // zero the other parity's group counters and active-list length for the next
-    // launch (the previous launch that used them has completed: same stream)
-    if (blockIdx.x == 0 && ctid == 0 && p.active_cnt_zero) {
-        *p.active_cnt_zero = 0u;
-        *p.nz_cnt_zero = 0u;
-    }
-    for (uint64_t k = (uint64_t)blockIdx.x * kConsumerThreads + ctid; k < p.n_group_zero;
-         k += (uint64_t)gridDim.x * kConsumerThreads)
-        p.group_zero[k] = 0;
-
-    ThreadAcc acc;
-    acc.reset();
-    int cur = -1;
-    SegHot g;
-
-    for (uint32_t i = 0;; ++i) {
-        const int s = i % S;
-        mbar_wait(&full_bar[s], (i / S) & 1);
-        const StageInfo si = info[s];
-        if (si.tile == ~0ull) break;
-        if ((int)si.seg != cur) {
-            const uint32_t slot = segs[si.seg].acc_slot;
-            if (cur >= 0 && slot != g.acc_slot) flush_acc(p.acc, g.acc_slot, g.dtype, acc, ctid, s_red_u, s_red_d);
-            cur = (int)si.seg;
-            g.load(segs[si.seg]);
-        }
-        const uint8_t *so = smem + (size_t)s * kStageBytes;
-        const uint32_t cnt = (p.flags & kFlagProbe) ? 0u : eval_any(so, so + kStageArrayBytes, si, ctid, g, acc);
-        acc.count += cnt;
-        if (g.max_report != 0) {
-            // Per-tile count for K2: warps fold their counts into the stage's
-            // shared word (arrivals << 24 | count); the last warp publishes the
-            // tile (2 global atomics per tile with mismatches, none otherwise)
-            // and clears the word before the stage can be reused.
-            const uint32_t wc = __reduce_add_sync(0xffffffffu, cnt);
-            if (lane == 0) {
-                const uint32_t old = atomicAdd(&s_tile[s], (1u << 24) | wc);
-                if ((old >> 24) == kConsumerWarps - 1) {
-                    const uint32_t tc = (old & 0xffffffu) + wc;
-                    s_tile[s] = 0u;
-                    if (tc != 0) {
-                        const uint64_t lt = si.tile - g.tile_begin;
-                        atomicAdd(p.tile_cnt + g.slot_begin + lt, tc);
-                        atomicAdd(p.group_cnt + g.group_begin + lt / kGroupTiles, tc);
-                        // short list of nonzero tiles for K2's pool path (checked
-                        // before the atomic so a dense call stops touching it)
-                        if (*(volatile uint32_t *)p.nz_cnt < (uint32_t)kPoolCap) {
-                            const uint32_t k = atomicAdd(p.nz_cnt, 1u);
-                            if (k < (uint32_t)kPoolCap) {
-                                p.nz_list[2 * k] = ((uint64_t)si.seg << 40) | lt;
-                                p.nz_list[2 * k + 1] = tc;
-                            }
-                        }
-                    }
-                }
-            }
-        }
-        if (p.flags & 1u) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&empty_bar[s]);  // stage may be refilled now
-    }
-    // K2 (programmatic dependent launch) may be scheduled from here on; it
-    // waits for this grid's completion before reading anything it wrote.
-    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-    if (cur >= 0) flush_acc(p.acc, g.acc_slot, g.dtype, acc, ctid, s_red_u, s_red_d);
-    // The last CTA publishes at once unless K2 has report entries to write: with
-    // no mismatch in any reporting region (the common "verified clean" case)
-    // the host wakes here while K2 -- then a no-op -- runs in the background.
-    if ((p.finalize || p.k2) && last_cta(p, ctid, kConsumerThreads, &s_last, false)) {
-        __threadfence();
-        if (p.finalize && (!p.k2 || *(volatile uint32_t *)p.nz_cnt == 0u)) publish(p, ctid, kConsumerThreads);
-    }
+                                                bool wrote_host, unsigned long long base, bool do_publish = true) {
+    if (last_cta(p, tid, nthreads, s_last, wrote_host, base) && do_publish) publish(p, tid, nthreads);
 }
 
 // --------------------------------------------------------------- K2 helpers
-// Exclusive block scan (256 threads, __syncthreads) of a u64; returns the
+// Exclusive scan over the 256 consumer threads (named barrier 1; `tid` = the
+// consumer index, so K1's consumer warps can run it too) of a u64; returns the
 // exclusive prefix, writes the block total to *total.
-__device__ __forceinline__ uint64_t block_excl_scan(uint64_t v, uint64_t *s_w, uint64_t *total) {
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+__device__ __forceinline__ uint64_t block_excl_scan(uint64_t v, uint64_t *s_w, uint64_t *total, int tid) {
+    const int lane = tid & 31, w = tid >> 5;
     uint64_t inc = v;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
@@ -708,7 +615,7 @@ __device__ __forceinline__ uint64_t block_excl_scan(uint64_t v, uint64_t *s_w, u
         if (lane >= o) inc += y;
     }
     if (lane == 31) s_w[w] = inc;
-    __syncthreads();
+    consumer_bar();
     uint64_t base = 0, tot = 0;
 #pragma unroll
     for (int k = 0; k < kConsumerWarps; ++k) {
@@ -716,7 +623,7 @@ __device__ __forceinline__ uint64_t block_excl_scan(uint64_t v, uint64_t *s_w, u
         base += (k < w) ? x : 0ull;
         tot += x;
     }
-    __syncthreads();
+    consumer_bar();
     *total = tot;
     return base + inc - v;
 }
@@ -725,16 +632,15 @@ __device__ __forceinline__ uint64_t block_excl_scan(uint64_t v, uint64_t *s_w, u
 // for ranks < max_report.  In-tile order = element index order = (k, tid, j).
 template <typename T>
 __device__ __noinline__ void compact_tile(const Seg &g, const StageInfo &si, const uint8_t *so, const uint8_t *sr,
-                                          uint64_t mask, uint64_t excl, uint64_t *s_w) {
+                                          uint64_t mask, uint64_t excl, uint64_t *s_w, int tid) {
     constexpr int EPV = 16 / sizeof(T);
     constexpr uint64_t kGroup = EPV == 64 ? ~0ull : ((1ull << EPV) - 1ull);
-    const int tid = threadIdx.x;
     uint64_t packed = 0;  // 4 x 16-bit per-k counts; field totals <= 4096 (no carries)
 #pragma unroll
     for (int k = 0; k < kVecPerThread; ++k)
         packed |= (uint64_t)__popcll(mask & (kGroup << (k * EPV))) << (16 * k);
     uint64_t total;
-    const uint64_t ex = block_excl_scan(packed, s_w, &total);
+    const uint64_t ex = block_excl_scan(packed, s_w, &total, tid);
     arc_mismatch_t *const rep = (excl & kDirectBit) ? g.report_alias : g.report;
     excl &= ~kDirectBit;
     uint64_t m = mask;
@@ -831,32 +737,39 @@ __device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long
 
 // Software grid barrier (K2 is launched cooperatively, so all CTAs are
 // co-resident).  Monotonic counter; the host tracks each launch's base.
-__device__ __forceinline__ void grid_barrier(unsigned long long *ctr, unsigned long long base) {
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        __threadfence();
+// `tid` = consumer index; the 256 consumer threads synchronise on barrier 1.
+__device__ __forceinline__ void grid_barrier(unsigned long long *ctr, unsigned long long base, int tid) {
+    consumer_bar();
+    if (tid == 0) {
+        fence_gpu();
         atomicAdd(ctr, 1ull);
-        while (ld_acquire_u64(ctr) - base < (unsigned long long)gridDim.x) __nanosleep(64);
+        while (ld_acquire_u64(ctr) - base < (unsigned long long)gridDim.x) __nanosleep(32);
     }
-    __syncthreads();
+    consumer_bar();
 }
 
 __device__ __forceinline__ void compact_any(const Seg &g, const StageInfo &si, const uint8_t *so, const uint8_t *sr,
-                                            uint64_t mask, uint64_t excl, uint64_t *s_w) {
+                                            uint64_t mask, uint64_t excl, uint64_t *s_w, int tid) {
     switch (g.dtype) {
-        case ARC_F32: compact_tile<float>(g, si, so, sr, mask, excl, s_w); break;
-        case ARC_F64: compact_tile<double>(g, si, so, sr, mask, excl, s_w); break;
-        case ARC_I32: compact_tile<int32_t>(g, si, so, sr, mask, excl, s_w); break;
-        case ARC_I64: compact_tile<int64_t>(g, si, so, sr, mask, excl, s_w); break;
-        default: compact_tile<uint8_t>(g, si, so, sr, mask, excl, s_w); break;
+        case ARC_F32: compact_tile<float>(g, si, so, sr, mask, excl, s_w, tid); break;
+        case ARC_F64: compact_tile<double>(g, si, so, sr, mask, excl, s_w, tid); break;
+        case ARC_I32: compact_tile<int32_t>(g, si, so, sr, mask, excl, s_w, tid); break;
+        case ARC_I64: compact_tile<int64_t>(g, si, so, sr, mask, excl, s_w, tid); break;
+        default: compact_tile<uint8_t>(g, si, so, sr, mask, excl, s_w, tid); break;
     }
 }
 
-// Two ways to find the tiles whose mismatches enter the report:
+// The report phase (a5): which tiles' mismatches enter the report, re-read them,
+// write their entries in ascending index order.  Runs either in K2 (its own
+// cooperative launch after K1) or -- fused, the default -- in K1's consumer
+// warps after a grid barrier, so the report costs no second launch.
+//
+// Two ways to find the report tiles:
 // Pool path (the common, sparse case: K1 listed <= kPoolCap nonzero tiles):
-//   every CTA loads the short list into shared memory; entry k (round-robin)
-//   gets its exclusive prefix = sum of counts of listed tiles of the same
-//   segment with a smaller index; no group walk, no grid barrier.
+//   pool entry k is handled by CTA k mod grid.  A CTA issues the bulk re-reads
+//   of its first two entries at once, then gets their exclusive prefixes in ONE
+//   pass over the pool (sum of the counts of listed tiles of the same segment
+//   with a smaller index; read from L2) and one block reduction; no grid barrier.
 // Group path (dense: the list overflowed):
 //   Phase A: every CTA scans the group counters of each reporting segment (a few
 //   KB); nonzero groups are owned round-robin by their ordinal, the owner scans
@@ -864,41 +777,37 @@ __device__ __forceinline__ void compact_any(const Seg &g, const StageInfo &si, c
 //   below max_report to the active list {seg, tile, prefix}.  Grid barrier.
 // Then each CTA re-reads its active tiles through a 2-stage bulk-copy ring,
 // re-evaluates them, and writes their mismatches at report positions
-// prefix + in-tile rank (ascending index order).  Tile counts are cleared for
-// the next call by whoever handled the tile / group.
-// grid: number of SMs (cooperative launch); block: 256;
-// dynamic smem: 2 stages + pool list (kPoolCap x 12 B).
-__global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __grid_constant__ Params p) {
-    extern __shared__ __align__(128) uint8_t smem[];
-    __shared__ __align__(8) uint64_t bar[2];
-    __shared__ uint64_t s_w[kConsumerWarps];
-    __shared__ uint32_t s_owned[kGroupTiles];
-    __shared__ uint64_t s_owned_pre[kGroupTiles];
-    __shared__ uint64_t s_loc_key[kPoolLocal];
-    __shared__ uint64_t s_loc_pre[kPoolLocal];
-    __shared__ uint32_t s_n;
-    __shared__ int s_last;
-    __shared__ int s_wrote;  // this CTA wrote report entries to pinned host memory
-    uint64_t *s_pkey = reinterpret_cast<uint64_t *>(smem + 2 * kStageBytes);
-    uint32_t *s_pcnt = reinterpret_cast<uint32_t *>(s_pkey + kPoolCap);
+// prefix + in-tile rank.  Tile counts are cleared for the next call by whoever
+// handled the tile / group.
+// `smem`: >= kReportSmem bytes of dynamic shared memory (2 stages + RepShared);
+// `tid`: consumer index 0..255 (named barrier 1).  Counter contract: adds
+// exactly gridDim.x to p.gbar, and (p.finalize) exactly gridDim.x to p.done
+// above `done_base`; the last CTA publishes unless `k1_published`.
+struct RepShared {
+    uint64_t bar[2];
+    uint64_t w[kConsumerWarps];
+    uint64_t red[kConsumerWarps][4];
+    uint64_t owned_pre[kGroupTiles];
+    uint32_t owned[kGroupTiles];
+    uint32_t n;
+    int last;
+    int wrote;  // this CTA wrote report entries to pinned host memory
+};
+constexpr int kReportSmem = 2 * kStageBytes + (int)sizeof(RepShared);
 
-    const Seg *segs = p.segs ? p.segs : p.inline_segs;
-    const int tid = threadIdx.x;
-    // launched as a programmatic dependent of K1: wait for K1's completion (and
-    // the visibility of its writes) before touching any of them
-    asm volatile("griddepcontrol.wait;" ::: "memory");
-    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");  // the exchange kernel, if any
+__device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, uint8_t *smem, int tid,
+                                             unsigned long long done_base, bool k1_published_if_empty) {
+    RepShared &sh = *reinterpret_cast<RepShared *>(smem + 2 * kStageBytes);
     if (tid == 0) {
-        s_wrote = 0;
-        mbar_init(&bar[0], 1);
-        mbar_init(&bar[1], 1);
+        ARCV_STAMP(1, 1);
+        sh.wrote = 0;
+        mbar_init(&sh.bar[0], 1);
+        mbar_init(&sh.bar[1], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
-    __syncthreads();
+    consumer_bar();
     const uint64_t policy = evict_first_policy();
     constexpr uint64_t kLtMask = (1ull << 40) - 1;
-
-    // re-read, re-evaluate and compact a list of active tiles {key, prefix}
     uint32_t phase[2] = {0u, 0u};
     auto issue = [&](uint64_t key, int st) {
         const Seg &g = segs[key >> 40];
@@ -907,98 +816,99 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
         uint32_t nbo, nbr;
         plan_tile(g, key & kLtMask, si, ao, nbo, ar, nbr);
         uint8_t *dst = smem + (size_t)st * kStageBytes;
-        mbar_arrive_expect_tx(&bar[st], nbo + nbr);
-        bulk_g2s(dst, reinterpret_cast<const void *>(ao), nbo, &bar[st], policy);
-        bulk_g2s(dst + kStageArrayBytes, reinterpret_cast<const void *>(ar), nbr, &bar[st], policy);
+        mbar_arrive_expect_tx(&sh.bar[st], nbo + nbr);
+        bulk_g2s(dst, reinterpret_cast<const void *>(ao), nbo, &sh.bar[st], policy);
+        bulk_g2s(dst + kStageArrayBytes, reinterpret_cast<const void *>(ar), nbr, &sh.bar[st], policy);
     };
-    auto process = [&](uint32_t n, auto get_key, auto get_pre) {
-        int st = 0;
-        if (n > 0 && tid == 0) issue(get_key(0u), 0);
-        for (uint32_t j = 0; j < n; ++j) {
-            if (j + 1 < n && tid == 0) issue(get_key(j + 1), st ^ 1);  // prefetch the next tile
-            const uint64_t key = get_key(j);
-            const uint64_t excl = get_pre(j);
-            const Seg &g = segs[key >> 40];
-            StageInfo si;
-            uintptr_t ao, ar;
-            uint32_t nbo, nbr;
-            plan_tile(g, key & kLtMask, si, ao, nbo, ar, nbr);
-            mbar_wait(&bar[st], phase[st]);
-            phase[st] ^= 1u;
+    // wait for tile `key` in stage st, write its entries from report rank excl
+    auto emit = [&](uint64_t key, uint64_t excl, int st, bool direct) {
+        const Seg &g = segs[key >> 40];
+        StageInfo si;
+        uintptr_t ao, ar;
+        uint32_t nbo, nbr;
+        plan_tile(g, key & kLtMask, si, ao, nbo, ar, nbr);
+        mbar_wait(&sh.bar[st], phase[st]);
+        phase[st] ^= 1u;
+        if (tid == 0) ARCV_STAMP(1, 4);
+        if (excl < g.max_report) {  // uniform
+            if ((direct || (g.flags & kSegReportHost)) && tid == 0) sh.wrote = 1;
             const uint8_t *so = smem + (size_t)st * kStageBytes;
-            SegHot gh;
-            gh.load(g);
-            const uint64_t mask = mask_any(so, so + kStageArrayBytes, si, tid, gh);
-            compact_any(g, si, so, so + kStageArrayBytes, mask, excl, s_w);
-            __syncthreads();  // stage `st` and s_w are reused
-            st ^= 1;
+            const uint64_t mask = mask_any(so, so + kStageArrayBytes, si, tid, g);
+            if (tid == 0) ARCV_STAMP(1, 5);
+            compact_any(g, si, so, so + kStageArrayBytes, mask, excl | (direct ? kDirectBit : 0ull), sh.w, tid);
         }
+        consumer_bar();  // stage `st` and sh.w are reused
+        if (tid == 0) ARCV_STAMP(1, 2);
     };
 
     const uint32_t n_nz = *(volatile uint32_t *)p.nz_cnt;
-    if (n_nz == 0) {
-        // nothing to report: K1 published; keep the grid-barrier and
-        // finished-CTA bookkeeping in step
-        if (tid == 0) atomicAdd(p.gbar, 1ull);
-        if (p.finalize) finalize_launch(p, tid, kConsumerThreads, &s_last, false, false);
-        return;
-    }
+    const uint32_t G = gridDim.x, b = blockIdx.x;
     if (n_nz <= (uint32_t)kPoolCap) {
         // ------------------------------------------------------ pool path
-        // arrive on the grid-barrier counter without waiting: the host advances
-        // its base by gridDim.x for every launch
+        // arrive on the grid-barrier counter without waiting (host base += grid)
         if (tid == 0) atomicAdd(p.gbar, 1ull);
-        for (uint32_t i = tid; i < n_nz; i += kConsumerThreads) {
-            s_pkey[i] = __ldcg(p.nz_list + 2 * i);
-            s_pcnt[i] = (uint32_t)__ldcg(p.nz_list + 2 * i + 1);
-        }
-        __syncthreads();
-        // This CTA's pool entries k = blockIdx.x + j * gridDim.x.  Their tile
-        // re-reads are issued first (two stages), so the copies' latency overlaps
-        // the prefix scans; an entry whose prefix is past max_report just drops
-        // its (completed) copy.
-        const uint32_t n_own = n_nz > blockIdx.x ? (n_nz - blockIdx.x + gridDim.x - 1) / gridDim.x : 0u;
+        const uint32_t n_own = n_nz > b ? (n_nz - b + G - 1) / G : 0u;
         if (tid == 0)
-            for (uint32_t j = 0; j < n_own && j < 2; ++j) issue(s_pkey[blockIdx.x + j * gridDim.x], (int)j);
-        for (uint32_t j = 0; j < n_own; ++j) {
-            const int st = (int)(j & 1);
-            const uint32_t k = blockIdx.x + j * gridDim.x;
-            const uint64_t key = s_pkey[k];
-            const uint64_t seg = key >> 40, lt = key & kLtMask;
-            uint64_t pre = 0, segtot = 0;
-            for (uint32_t i = tid; i < n_nz; i += kConsumerThreads) {
-                const uint64_t ki = s_pkey[i];
-                if ((ki >> 40) == seg) {
-                    segtot += s_pcnt[i];
-                    pre += ((ki & kLtMask) < lt) ? s_pcnt[i] : 0u;
-                }
+            for (uint32_t j = 0; j < n_own && j < 2; ++j) issue(__ldcg(p.nz_list + 2 * (b + j * G)), (int)j);
+        // the whole pool in registers, all loads in flight at once: entry
+        // tid + u * 256 = {seg << 40 | tile, count}; absent entries never match
+        constexpr int kPer = kPoolCap / kConsumerThreads;
+        uint64_t pk[kPer], pc[kPer];
+#pragma unroll
+        for (int u = 0; u < kPer; ++u) {
+            const uint32_t i = (uint32_t)tid + (uint32_t)u * kConsumerThreads;
+            ulonglong2 e = make_ulonglong2(~0ull, 0ull);
+            if (i < n_nz) e = __ldcg(reinterpret_cast<const ulonglong2 *>(p.nz_list) + i);
+            pk[u] = e.x;
+            pc[u] = e.y;
+        }
+        for (uint32_t j0 = 0; j0 < n_own; j0 += 2) {
+            const uint32_t m = n_own - j0 < 2u ? n_own - j0 : 2u;
+            uint64_t key[2], pre[2] = {0, 0}, tot[2] = {0, 0};
+            key[0] = __ldcg(p.nz_list + 2 * (b + j0 * G));
+            key[1] = m > 1 ? __ldcg(p.nz_list + 2 * (b + (j0 + 1) * G)) : ~0ull - 1;
+#pragma unroll
+            for (int u = 0; u < kPer; ++u)
+#pragma unroll
+                for (int q = 0; q < 2; ++q)
+                    if ((pk[u] >> 40) == (key[q] >> 40)) {
+                        tot[q] += pc[u];
+                        pre[q] += (pk[u] & kLtMask) < (key[q] & kLtMask) ? pc[u] : 0ull;
+                    }
+#pragma unroll
+            for (int q = 0; q < 2; ++q) {
+                pre[q] = warp_sum_u64(pre[q]);
+                tot[q] = warp_sum_u64(tot[q]);
             }
-            uint64_t pre_tot, seg_tot;
-            block_excl_scan(pre, s_w, &pre_tot);
-            block_excl_scan(segtot, s_w, &seg_tot);
-            const Seg &g = segs[seg];
-            uint64_t base = 0;
-            if (g.flags & kSegBaseFromAcc) base = __ldcg(&p.acc[g.acc_slot].count) - seg_tot;
-            const uint64_t excl = base + pre_tot;
-            if (tid == 0) p.tile_cnt[g.slot_begin + lt] = 0u;  // clean for the next call
-            mbar_wait(&bar[st], phase[st]);
-            phase[st] ^= 1u;
-            if (excl < g.max_report) {  // uniform
+            if ((tid & 31) == 0) {
+                sh.red[tid >> 5][0] = pre[0];
+                sh.red[tid >> 5][1] = pre[1];
+                sh.red[tid >> 5][2] = tot[0];
+                sh.red[tid >> 5][3] = tot[1];
+            }
+            consumer_bar();
+            uint64_t r[4] = {0, 0, 0, 0};
+#pragma unroll
+            for (int w = 0; w < kConsumerWarps; ++w)
+#pragma unroll
+                for (int c = 0; c < 4; ++c) r[c] += sh.red[w][c];
+            if (tid == 0) ARCV_STAMP(1, 3);
+            for (uint32_t q = 0; q < m; ++q) {
+                const uint32_t j = j0 + q;
+                const int st = (int)(j & 1);
+                const Seg &g = segs[key[q] >> 40];
+                const uint64_t seg_tot = r[2 + q];
+                uint64_t base = 0;
+                if (g.flags & kSegBaseFromAcc) base = __ldcg(&p.acc[g.acc_slot].count) - seg_tot;
+                if (tid == 0) p.tile_cnt[g.slot_begin + (key[q] & kLtMask)] = 0u;  // clean for the next call
                 // a sparse region with a pinned host report: written over PCIe
                 // directly (the host then skips its D2H copy; same rule there)
                 const bool direct = g.report_alias && !(g.flags & kSegBaseFromAcc) && seg_tot <= kDirectDyn;
-                if (direct && tid == 0) s_wrote = 1;
-                StageInfo si;
-                uintptr_t ao, ar;
-                uint32_t nbo, nbr;
-                plan_tile(g, lt, si, ao, nbo, ar, nbr);
-                const uint8_t *so = smem + (size_t)st * kStageBytes;
-                const uint64_t mask = mask_any(so, so + kStageArrayBytes, si, tid, g);
-                compact_any(g, si, so, so + kStageArrayBytes, mask, excl | (direct ? kDirectBit : 0ull), s_w);
+                emit(key[q], base + r[q], st, direct);  // ends with a barrier: sh.red free again
+                if (tid == 0 && j + 2 < n_own) issue(__ldcg(p.nz_list + 2 * (b + (j + 2) * G)), st);
             }
-            __syncthreads();  // stage `st` and s_w are reused
-            if (tid == 0 && j + 2 < n_own) issue(s_pkey[k + 2 * gridDim.x], st);
         }
+        if (tid == 0) ARCV_STAMP(1, 6);
     } else {
         // ------------------------------------------------------ group path
         for (uint32_t sgi = 0; sgi < p.n_segs; ++sgi) {
@@ -1010,7 +920,7 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
             uint64_t tot = 0;
             for (uint64_t k = tid; k < ngroups; k += kConsumerThreads) tot += __ldcg(gc + k);
             uint64_t total;
-            block_excl_scan(tot, s_w, &total);
+            block_excl_scan(tot, sh.w, &total, tid);
             if (total == 0) continue;  // uniform: nothing to report or to clear
             uint64_t base = 0;
             if (g.flags & kSegBaseFromAcc) base = __ldcg(&p.acc[g.acc_slot].count) - total;
@@ -1022,29 +932,29 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
                 // pack (nonzero ordinal, count): group counts < 2^23, 256 of them < 2^31
                 const uint64_t v = ((uint64_t)(cnt != 0) << 40) | cnt;
                 uint64_t ctot;
-                const uint64_t ex = block_excl_scan(v, s_w, &ctot);
+                const uint64_t ex = block_excl_scan(v, sh.w, &ctot, tid);
                 const uint64_t gpre = run + (ex & ((1ull << 40) - 1));
                 const uint64_t ord = ord_run + (ex >> 40);
-                if (tid == 0) s_n = 0;
-                __syncthreads();
-                if (cnt != 0 && (ord % gridDim.x) == blockIdx.x) {
-                    const uint32_t k = atomicAdd(&s_n, 1u);
-                    s_owned[k] = (uint32_t)gi;
-                    s_owned_pre[k] = gpre;
+                if (tid == 0) sh.n = 0;
+                consumer_bar();
+                if (cnt != 0 && (ord % G) == b) {
+                    const uint32_t k = atomicAdd(&sh.n, 1u);
+                    sh.owned[k] = (uint32_t)gi;
+                    sh.owned_pre[k] = gpre;
                 }
-                __syncthreads();
-                const uint32_t n_owned = s_n;
+                consumer_bar();
+                const uint32_t n_owned = sh.n;
                 run += ctot & ((1ull << 40) - 1);
                 ord_run += ctot >> 40;
                 for (uint32_t q = 0; q < n_owned; ++q) {
-                    const uint64_t t0 = (uint64_t)s_owned[q] * kGroupTiles;
-                    const uint64_t gp = s_owned_pre[q];
+                    const uint64_t t0 = (uint64_t)sh.owned[q] * kGroupTiles;
+                    const uint64_t gp = sh.owned_pre[q];
                     const uint64_t tg = ntiles - t0 < (uint64_t)kGroupTiles ? ntiles - t0 : (uint64_t)kGroupTiles;
                     uint32_t *tc = p.tile_cnt + g.slot_begin + t0;
                     const uint32_t tcnt = (uint64_t)tid < tg ? __ldcg(tc + tid) : 0u;
                     if (gp < g.max_report) {  // uniform
                         uint64_t gtot;
-                        const uint64_t tpre = gp + block_excl_scan(tcnt, s_w, &gtot);
+                        const uint64_t tpre = gp + block_excl_scan(tcnt, sh.w, &gtot, tid);
                         if (tcnt != 0 && tpre < g.max_report) {
                             const uint32_t k = atomicAdd(p.active_cnt, 1u);
                             p.active[2 * k] = ((uint64_t)sgi << 40) | (t0 + tid);
@@ -1053,16 +963,206 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
                     }
                     if (tcnt != 0) tc[tid] = 0u;  // clean for the next call
                 }
-                __syncthreads();
+                consumer_bar();
             }
         }
-        grid_barrier(p.gbar, p.gbar_base);
+        grid_barrier(p.gbar, p.gbar_base, tid);
         const uint32_t n_act = *(volatile uint32_t *)p.active_cnt;
-        const uint32_t mine = n_act > blockIdx.x ? (n_act - blockIdx.x + gridDim.x - 1) / gridDim.x : 0u;
-        process(mine, [&](uint32_t j) { return __ldcg(p.active + 2 * (blockIdx.x + j * gridDim.x)); },
-                [&](uint32_t j) { return __ldcg(p.active + 2 * (blockIdx.x + j * gridDim.x) + 1); });
+        const uint32_t mine = n_act > b ? (n_act - b + G - 1) / G : 0u;
+        if (mine > 0 && tid == 0) issue(__ldcg(p.active + 2 * b), 0);
+        for (uint32_t j = 0; j < mine; ++j) {
+            const int st = (int)(j & 1);
+            if (j + 1 < mine && tid == 0) issue(__ldcg(p.active + 2 * (b + (j + 1) * G)), st ^ 1);  // prefetch
+            const uint64_t key = __ldcg(p.active + 2 * (b + j * G));
+            const uint64_t excl = __ldcg(p.active + 2 * (b + j * G) + 1);
+            emit(key, excl, st, false);
+        }
     }
-    if (p.finalize) finalize_launch(p, tid, kConsumerThreads, &s_last, p.report_host != 0 || s_wrote != 0);
+    // Report entries in pinned host memory need no system-scope fence here:
+    // this CTA's gpu-scope release (fence + done counter) is acquired by the
+    // last CTA, whose fence.acq_rel.sys before the completion word is
+    // cumulative -- every write that happens-before it (these entries
+    // included) is visible to the host that acquires the word.  One PCIe
+    // flush per call instead of one per writing CTA.
+    // (-DARCV_WRITER_SYS=1: a system-scope fence in every writing CTA.)
+#if defined(ARCV_WRITER_SYS) && ARCV_WRITER_SYS
+    const bool wrote_host = p.report_host != 0 || sh.wrote != 0;
+#else
+    const bool wrote_host = false;
+#endif
+    if (p.finalize)
+        finalize_launch(p, tid, kConsumerThreads, &sh.last, wrote_host, done_base,
+                        !(k1_published_if_empty && n_nz == 0));
+    if (tid == 0) ARCV_STAMP(1, 7);
 }
+
+// K2: the report phase as its own launch (cooperative: the group path has a
+// grid barrier), a programmatic dependent of K1.  Used when the fused tail does
+// not fit K1's stage memory (fewer than 3 stages) or ARCV_FUSED=0.
+// grid: SMs x co-resident CTAs; block: 256; dynamic smem: kReportSmem.
+__global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __grid_constant__ Params p) {
+    extern __shared__ __align__(128) uint8_t smem[];
+    const Seg *segs = p.segs ? p.segs : p.inline_segs;
+    if (threadIdx.x == 0) ARCV_STAMP(1, 0);
+    // wait for K1's completion (and the visibility of its writes) before
+    // touching any of them
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");  // the exchange kernel, if any
+    report_phase(p, segs, smem, (int)threadIdx.x, p.done_base, true);
+}
+
+
+// ------------------------------------------------------------------ K1: stream
+template <int S, int MINB>
+__global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __grid_constant__ Params p) {
+    extern __shared__ __align__(128) uint8_t smem[];
+    __shared__ __align__(8) uint64_t full_bar[S];
+    __shared__ __align__(8) uint64_t empty_bar[S];
+    __shared__ StageInfo info[S];
+    __shared__ uint64_t s_red_u[kConsumerWarps][2];
+    __shared__ double s_red_d[kConsumerWarps][2];
+    __shared__ int s_last;
+    __shared__ uint32_t s_tile[S];
+
+    const Seg *segs = p.segs ? p.segs : p.inline_segs;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < S; ++s) {
+            s_tile[s] = 0u;
+            mbar_init(&full_bar[s], 1);
+            mbar_init(&empty_bar[s], kConsumerWarps);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+
+    // ------------------------------------------------------------ producer
+    if (warp == 0) {
+        if (lane == 0) {
+            const uint64_t policy = evict_first_policy();
+            for (uint32_t i = 0;; ++i) {
+                const int s = i % S;
+                if (i >= (uint32_t)S) mbar_wait(&empty_bar[s], ((i / S) - 1) & 1);
+                const uint64_t t = atomicAdd(p.ticket, 1ull) - p.ticket_base;
+                if (t >= p.total_tiles) {
+                    info[s].tile = ~0ull;
+                    mbar_arrive(&full_bar[s]);
+                    break;
+                }
+                const uint32_t sg = find_seg(segs, p.n_segs, t);
+                const Seg &g = segs[sg];
+                StageInfo &si = info[s];
+                uintptr_t ao, ar;
+                uint32_t nbo, nbr;
+                plan_tile(g, t - g.tile_begin, si, ao, nbo, ar, nbr);
+                si.tile = t;
+                si.seg = sg;
+                uint8_t *dst = smem + (size_t)s * kStageBytes;
+                mbar_arrive_expect_tx(&full_bar[s], nbo + nbr);
+                bulk_g2s(dst, reinterpret_cast<const void *>(ao), nbo, &full_bar[s], policy);
+                bulk_g2s(dst + kStageArrayBytes, reinterpret_cast<const void *>(ar), nbr, &full_bar[s], policy);
+            }
+        }
+        return;
+    }
+
+    // ------------------------------------------------------------ consumers
+    const int ctid = threadIdx.x - 32;
+    // zero the other parity's group counters and active-list length for the next
+    // launch (the previous launch that used them has completed: same stream)
+    if (blockIdx.x == 0 && ctid == 0 && p.active_cnt_zero) {
+        *p.active_cnt_zero = 0u;
+        *p.nz_cnt_zero = 0u;
+    }
+    for (uint64_t k = (uint64_t)blockIdx.x * kConsumerThreads + ctid; k < p.n_group_zero;
+         k += (uint64_t)gridDim.x * kConsumerThreads)
+        p.group_zero[k] = 0;
+
+    ThreadAcc acc;
+    acc.reset();
+    int cur = -1;
+    SegHot g;
+    if (ctid == 0) ARCV_STAMP(0, 0);
+
+    for (uint32_t i = 0;; ++i) {
+        const int s = i % S;
+        mbar_wait(&full_bar[s], (i / S) & 1);
+        const StageInfo si = info[s];
+        if (si.tile == ~0ull) break;
+        if ((int)si.seg != cur) {
+            const uint32_t slot = segs[si.seg].acc_slot;
+            if (cur >= 0 && slot != g.acc_slot) flush_acc(p.acc, g.acc_slot, g.dtype, acc, ctid, s_red_u, s_red_d);
+            cur = (int)si.seg;
+            g.load(segs[si.seg]);
+        }
+        const uint8_t *so = smem + (size_t)s * kStageBytes;
+        const uint32_t cnt = (p.flags & kFlagProbe) ? 0u : eval_any(so, so + kStageArrayBytes, si, ctid, g, acc);
+        acc.count += cnt;
+        if (g.max_report != 0) {
+            // Per-tile count for K2: warps fold their counts into the stage's
+            // shared word (arrivals << 24 | count); the last warp publishes the
+            // tile (2 global atomics per tile with mismatches, none otherwise)
+            // and clears the word before the stage can be reused.
+            const uint32_t wc = __reduce_add_sync(0xffffffffu, cnt);
+            if (lane == 0) {
+                const uint32_t old = atomicAdd(&s_tile[s], (1u << 24) | wc);
+                if ((old >> 24) == kConsumerWarps - 1) {
+                    const uint32_t tc = (old & 0xffffffu) + wc;
+                    s_tile[s] = 0u;
+                    if (tc != 0) {
+                        const uint64_t lt = si.tile - g.tile_begin;
+                        atomicAdd(p.tile_cnt + g.slot_begin + lt, tc);
+                        atomicAdd(p.group_cnt + g.group_begin + lt / kGroupTiles, tc);
+                        // short list of nonzero tiles for K2's pool path (checked
+                        // before the atomic so a dense call stops touching it)
+                        if (*(volatile uint32_t *)p.nz_cnt < (uint32_t)kPoolCap) {
+                            const uint32_t k = atomicAdd(p.nz_cnt, 1u);
+                            if (k < (uint32_t)kPoolCap) {
+                                p.nz_list[2 * k] = ((uint64_t)si.seg << 40) | lt;
+                                p.nz_list[2 * k + 1] = tc;
+                            }
+                        }
+                    }
+                }
+            }
+        }
+        if (p.flags & 1u) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&empty_bar[s]);  // stage may be refilled now
+    }
+    // K2 (programmatic dependent launch) may be scheduled from here on; it
+    // waits for this grid's completion before reading anything it wrote.
+    if (ctid == 0) ARCV_STAMP(0, 1);
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    if (cur >= 0) flush_acc(p.acc, g.acc_slot, g.dtype, acc, ctid, s_red_u, s_red_d);
+    if (ctid == 0) ARCV_STAMP(0, 2);
+    if constexpr (S * kStageBytes >= kReportSmem) {
+        if (p.fused) {
+            // Fused report phase (cooperative launch: every CTA is resident).
+            // Grid barrier on the done counter: the tile counts and the pool
+            // are complete once every CTA has flushed.  The stage memory is
+            // free (the sentinel stage follows every real fill).
+            if (ctid == 0) {
+                ARCV_STAMP(1, 0);
+                fence_gpu();
+                atomicAdd(p.done, 1ull);
+                while (ld_acquire_u64(p.done) - p.done_base < (unsigned long long)gridDim.x) __nanosleep(32);
+            }
+            consumer_bar();
+            report_phase(p, segs, smem, ctid, p.done_base + gridDim.x, false);
+            return;
+        }
+    }
+    // The last CTA publishes at once unless K2 has report entries to write: with
+    // no mismatch in any reporting region (the common "verified clean" case)
+    // the host wakes here while K2 -- then a no-op -- runs in the background.
+    if ((p.finalize || p.k2) && last_cta(p, ctid, kConsumerThreads, &s_last, false, p.done_base)) {
+        fence_gpu();
+        if (p.finalize && (!p.k2 || *(volatile uint32_t *)p.nz_cnt == 0u)) publish(p, ctid, kConsumerThreads);
+    }
+    if (ctid == 0) ARCV_STAMP(0, 3);
+}
+
 
 }  // namespace arcv

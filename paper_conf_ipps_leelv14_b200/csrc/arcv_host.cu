@@ -114,7 +114,7 @@ PtrKind classify(const void *p, int device) {
     }
 }
 
-constexpr int kCompactSmem = 2 * kStageBytes + kPoolCap * (8 + 4);
+constexpr int kCompactSmem = kReportSmem;
 
 // Pinned host reports with a capacity up to Ctx::direct_max entries are
 // written by the kernel over PCIe; larger ones are staged in HBM and copied
@@ -234,6 +234,11 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
     int st = ARC_OK;
     Params p;
     memset(&p, 0, sizeof(p));
+    for (uint32_t k = 0; k < n_segs; ++k)
+        if (segs[k].report && classify(segs[k].report, c.device) != PK_DEVICE) {
+            p.report_host = 1;
+            segs[k].flags |= kSegReportHost;
+        }
     if (n_segs <= (uint32_t)kMaxInlineSegs) {
         memcpy(p.inline_segs, segs, n_segs * sizeof(Seg));
         p.segs = nullptr;
@@ -275,21 +280,44 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
     p.done_flag = ((c.flags & 8) || c.defer_wait) ? nullptr : c.flag_dev;
     if (finalize) p.seq = ++c.seq;  // the host waits for the last finalize launch's number
     p.mirror = finalize ? c.mirror_next : nullptr;
-    for (uint32_t k = 0; k < n_segs; ++k)
-        if (segs[k].report && classify(segs[k].report, c.device) != PK_DEVICE) p.report_host = 1;
 
     const uint64_t max_grid = (uint64_t)c.num_sms * (uint64_t)c.ctas_per_sm;
     const uint32_t grid = (uint32_t)std::min<uint64_t>(tiles, max_grid);
     const size_t smem = (size_t)c.stages * kStageBytes;
     const bool timed = c.timing && c.n_ev < Ctx::kMaxEv;
+    // fused: K1 runs the report phase after a grid barrier (cooperative launch)
+    const bool fused = need_compact && c.fused;
+    p.fused = fused ? 1 : 0;
     if (timed) CK(cudaEventRecord(c.ev[c.n_ev][0], c.stream));
-    stream_kernel_for(c.stages)<<<grid, kThreads, smem, c.stream>>>(p);
-    cudaError_t e = cudaGetLastError();
-    if (e != cudaSuccess) return cuda_fail(e, "arcv_stream_kernel launch");
+    cudaError_t e;
+    if (fused) {
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(grid);
+        cfg.blockDim = dim3(kThreads);
+        cfg.dynamicSmemBytes = smem;
+        cfg.stream = c.stream;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeCooperative;
+        at[0].val.cooperative = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        e = cudaLaunchKernelEx(&cfg, stream_kernel_for(c.stages), p);
+        if (e != cudaSuccess) return cuda_fail(e, "arcv_stream_kernel cooperative launch");
+    } else {
+        stream_kernel_for(c.stages)<<<grid, kThreads, smem, c.stream>>>(p);
+        e = cudaGetLastError();
+        if (e != cudaSuccess) return cuda_fail(e, "arcv_stream_kernel launch");
+    }
     c.launches++;
     c.ticket_base += tiles + grid;
-    if (p.finalize || p.k2) c.done_base += grid;  // K1 counts its CTAs to find its last one
-    if (need_compact) {
+    if (fused) {
+        // grid barrier + (finalize) the report phase's completion count
+        c.done_base += (uint64_t)grid * (finalize ? 2u : 1u);
+        c.gbar_base += grid;
+    } else if (p.finalize || p.k2) {
+        c.done_base += grid;  // K1 counts its CTAs to find its last one
+    }
+    if (need_compact && !fused) {
         p.finalize = finalize ? 1 : 0;
         p.done_base = c.done_base;
         const uint32_t grid2 = (uint32_t)c.k2_grid;
@@ -621,11 +649,6 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
     c->rank = o.rank;
     c->nranks = o.nranks;
     c->num_sms = prop.multiProcessorCount;
-    if (c->num_sms * kPoolLocal < kPoolCap) {  // K2 pool path: per-CTA share must fit
-        set_error("device has %d SMs; need >= %d", c->num_sms, kPoolCap / kPoolLocal);
-        delete c;
-        return ARC_E_UNSUPPORTED;
-    }
     if (o.stream) {
         c->stream = static_cast<cudaStream_t>(o.stream);
         c->own_stream = false;
@@ -665,11 +688,14 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
     c->k2_grid = c->num_sms * std::max(1, std::min(occ2, k2cap > 0 ? k2cap : 1));
     const int cap = env_int("ARCV_CTAS_PER_SM", 0);
     c->ctas_per_sm = cap > 0 ? std::min(cap, occ) : occ;
+    // the report phase runs in K1's tail when its stage memory holds the
+    // report phase's (>= 3 stages); ARCV_FUSED=0 forces the separate K2
+    c->fused = env_int("ARCV_FUSED", 1) != 0 && smem >= (size_t)kReportSmem;
     if (env_int("ARCV_VERBOSE", 0)) {
         cudaFuncAttributes fa;
         CK(cudaFuncGetAttributes(&fa, kf));
-        fprintf(stderr, "[arcv] sms=%d stages=%d ctas/sm=%d (occupancy %d) k2_grid=%d regs=%d static_smem=%zu dyn_smem=%zu local=%zu\n",
-                c->num_sms, c->stages, c->ctas_per_sm, occ, c->k2_grid, fa.numRegs, fa.sharedSizeBytes, smem, fa.localSizeBytes);
+        fprintf(stderr, "[arcv] sms=%d stages=%d ctas/sm=%d (occupancy %d) k2_grid=%d fused=%d regs=%d static_smem=%zu dyn_smem=%zu local=%zu\n",
+                c->num_sms, c->stages, c->ctas_per_sm, occ, c->k2_grid, (int)c->fused, fa.numRegs, fa.sharedSizeBytes, smem, fa.localSizeBytes);
     }
     // counters: [0] tile tickets, [1] finished CTAs, [2] K2 grid barrier,
     // [3] 2 x u32 active-list lengths, [4] 2 x u32 pool lengths (by parity),
@@ -801,6 +827,23 @@ int arc_verify_compare_ex(const void *out, const void *ref, uint64_t n, arc_dtyp
     r.check = (check && check->flags) ? check : nullptr;
     if (g_ctx->sharded) return shard_compare(*g_ctx, r, result);
     return run_local(*g_ctx, &r, 1, result, nullptr, true, nullptr);
+}
+
+// Diagnostic (A/B builds with -DARCV_TRACE=1 only): copy the per-CTA phase
+// stamps of the last traced launch pair, [2][1024][12] u64, into `out`.
+extern "C" int arc_verify_debug_trace(unsigned long long *out) {
+#if defined(ARCV_TRACE) && ARCV_TRACE
+    if (!g_ctx) return ARC_E_NOINIT;
+    CK(cudaStreamSynchronize(g_ctx->stream));
+    CK(cudaMemcpyFromSymbol(out, arcv::g_trace, sizeof(arcv::g_trace)));
+    std::vector<unsigned long long> zero(sizeof(arcv::g_trace) / 8, 0ull);
+    CK(cudaMemcpyToSymbol(arcv::g_trace, zero.data(), sizeof(arcv::g_trace)));
+    return ARC_OK;
+#else
+    (void)out;
+    set_error("built without ARCV_TRACE");
+    return ARC_E_UNSUPPORTED;
+#endif
 }
 
 int arc_verify_probe_read(const void *a, const void *b, uint64_t bytes, int iters, double *gbs) {

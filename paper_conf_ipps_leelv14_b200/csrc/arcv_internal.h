@@ -23,6 +23,7 @@ struct Ctx {
     int num_sms = 0, ctas_per_sm = 1, stages = 3, flags = 0;
     int k2_grid = 0;  // K2 (cooperative) grid: SMs x co-resident CTAs (<= 2)
     uint64_t direct_max = 0;  // pinned host reports up to this capacity: written by the kernel
+    bool fused = true;  // report phase in K1's tail (cooperative K1), no K2 launch
     bool pdl = true;  // launch K2 / the exchange kernel as programmatic dependents (ARCV_PDL=0: off)
     cudaStream_t stream = nullptr;
     bool own_stream = false;

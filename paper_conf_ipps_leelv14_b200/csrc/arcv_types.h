@@ -17,7 +17,6 @@ constexpr int kVecPerThread = kTileBytes / 16 / kConsumerThreads;  // 4
 constexpr int kMaxInlineSegs = 8;
 constexpr int kGroupTiles = 256;                    // tiles per group counter
 constexpr int kPoolCap = 2048;                      // K2 pool path: max listed nonzero tiles
-constexpr int kPoolLocal = 64;                      // per-CTA share of the pool (grid >= 32)
 constexpr uint64_t kDirectDyn = 4096;               // sparse reports: K2 writes a pinned host report directly
 constexpr uint64_t kDirectBit = 1ull << 63;         // K2 tile prefix flag: entries go to report_alias
 static_assert(kVecPerThread == 4, "packed-scan layout assumes 4 vectors per thread");
@@ -25,6 +24,7 @@ static_assert(kGroupTiles == kConsumerThreads, "K2 scans one group per block pas
 
 constexpr uint32_t kFlagProbe = 2u;       // Params.flags: stream only, no predicate (read probe)
 constexpr uint32_t kSegBaseFromAcc = 1u;  // chunk of a streamed region: prefix base = acc count - own total
+constexpr uint32_t kSegReportHost = 2u;   // `report` is (mapped) host memory: K2's writes need a system-scope release
 
 // One contiguous piece of one region (a whole region, or one chunk of a region
 // streamed from host memory).
@@ -77,6 +77,7 @@ struct Params {
     uint32_t *nz_cnt;         // this launch's pool length (may exceed kPoolCap: overflow)
     uint32_t *nz_cnt_zero;    // the other parity
     int k2;                   // K2 follows this K1 (some segment wants a report)
+    int fused;                // K1 runs the report phase itself (cooperative launch; no K2)
     unsigned long long *gbar; // K2 grid barrier counter (monotonic)
     unsigned long long gbar_base;
     Acc *acc;

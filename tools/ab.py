@@ -141,6 +141,14 @@ def c4():
     return single(o, r, c.abs_tol, c.rel_tol, c.max_report)
 
 
+def c4shard(lg):
+    def f():
+        c = synth.C4(1 << lg)
+        o, r = c.slice(device="cuda")
+        return single(o, r, c.abs_tol, c.rel_tol, c.max_report)
+    return f
+
+
 def i32clean():
     reg = synth.configs.Region("I", "i32", 1 << 28, 78, 0, 0, 1 << 20, "i32")
     o, r = reg.slice(device="cuda")
@@ -167,6 +175,8 @@ add("C3batch", c3)
 add("i32clean_2^28", i32clean)
 add("u8clean_2^30", u8clean)
 add("C4", c4)
+add("C4_2^26", c4shard(26))
+add("C4_2^27", c4shard(27))
 add("C5", c5)
 
 print(f"libs: {libs}; rounds {ROUNDS} x {STEPS} steps", flush=True)
