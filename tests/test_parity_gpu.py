@@ -259,14 +259,16 @@ def test_host_inputs_streamed(av, orc, where):
 
 
 # ------------------------------------------------------------ stage variants
-@pytest.mark.parametrize("stages,ctas,flags", [(2, 0, 0), (4, 0, 0), (6, 0, 0), (3, 1, 0), (3, 0, 8)])
-def test_launch_geometry_invariance(orc, stages, ctas, flags):
-    """Stage counts, CTAs per SM, and (flags=8) stream-sync instead of the completion word."""
+@pytest.mark.parametrize("stages,ctas,flags,fused", [(2, 0, 0, 1), (4, 0, 0, 1), (6, 0, 0, 1), (3, 1, 0, 1),
+                                                     (3, 0, 8, 1), (3, 0, 0, 0), (4, 1, 0, 0)])
+def test_launch_geometry_invariance(orc, stages, ctas, flags, fused):
+    """Stage counts, CTAs per SM, (flags=8) stream-sync instead of the completion word, and
+    (fused=0, or 2 stages) the report phase as its own launch (K2) instead of K1's tail."""
     import paper_conf_ipps_leelv14_b200 as av
 
     av.finalize()
     os.environ["ARCV_STAGES"], os.environ["ARCV_CTAS_PER_SM"] = str(stages), str(ctas)
-    os.environ["ARCV_FLAGS"] = str(flags)
+    os.environ["ARCV_FLAGS"], os.environ["ARCV_FUSED"] = str(flags), str(fused)
     try:
         av.init(0)
         c1 = synth.C1()
@@ -281,7 +283,26 @@ def test_launch_geometry_invariance(orc, stages, ctas, flags):
     finally:
         av.finalize()
         del os.environ["ARCV_STAGES"], os.environ["ARCV_CTAS_PER_SM"], os.environ["ARCV_FLAGS"]
+        del os.environ["ARCV_FUSED"]
         av.init(0)
+
+
+@pytest.mark.parametrize("n_tiles", [1, 295, 296, 297, 2047, 2048, 2049])
+def test_pool_capacity_boundary(av, orc, n_tiles):
+    """One mismatch in each of `n_tiles` distinct tiles: up to 2048 nonzero tiles the report
+    phase takes the pool path (several entries per CTA beyond 296), from 2049 the group path."""
+    te = TILE_ELEMS["f32"]
+    n = 4096 * te + 777  # ragged tail tile
+    gen = torch.Generator(device="cpu").manual_seed(7000 + n_tiles)
+    ref = (torch.rand(n, generator=gen, dtype=torch.float64) + 0.5).to(torch.float32)
+    out = ref.clone()
+    tiles = torch.randperm(4097, generator=gen)[:n_tiles]
+    pos = torch.randint(0, 777, (n_tiles,), generator=gen)  # valid in the tail tile too
+    idx = tiles * te + pos
+    out[idx] = out[idx] + 1.0
+    out, ref = out.cuda(), ref.cuda()
+    for mr in (1, n_tiles // 2 + 1, n_tiles, 1 << 20):
+        run_both(av, orc, out, ref, "f32", 1e-6, 1e-5, mr, f"tiles={n_tiles} mr={mr}")
 
 
 # --------------------------------------------------------------- full sizes

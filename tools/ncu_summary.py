@@ -33,10 +33,10 @@ def main():
             out[name] = one(f"gpurun_out/{tag}_{name}_raw.csv")
         except (OSError, IndexError):
             pass
-    try:
-        k1, k2 = out["k1_c4"], out["k2_c4"]
-        b = lambda s, u: float(s.split()[0]) * {"Gbyte": 1e9, "Mbyte": 1e6, "Kbyte": 1e3, "byte": 1}[s.split()[1]]
-        out["c4_dram_bytes_per_launch"] = int(sum(b(k[m], None) for k in (k1, k2)
+    try:  # per call: K1 (with the fused report phase), + K2 when it was a separate launch
+        ks = [out[k] for k in ("k1_c4", "k2_c4") if k in out]
+        b = lambda s: float(s.split()[0]) * {"Gbyte": 1e9, "Mbyte": 1e6, "Kbyte": 1e3, "byte": 1}[s.split()[1]]
+        out["c4_dram_bytes_per_launch"] = int(sum(b(k[m]) for k in ks
                                                   for m in ("dram__bytes_read.sum", "dram__bytes_write.sum")))
     except (KeyError, ValueError, IndexError):
         pass

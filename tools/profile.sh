@@ -3,7 +3,7 @@
 #   bash tools/profile.sh TAG
 # 1. launch list of the bench command (per-launch gpu__time_duration, cold
 #    cache, serialised -- the kernels' SHARE of a step, not a bench number);
-# 2. one `--set full` capture of K1 and of K2 on the bench workload (C4);
+# 2. one `--set full` capture of K1 (stream + fused report phase) on the bench workload (C4);
 # 3. one `--set full` capture of K1 on C2A (Jacobi-2D 8192^2 fp32, clean).
 set -u
 TAG=${1:-prof}
@@ -15,9 +15,6 @@ echo "launches rc=$?"
 $NCU --set full --clock-control none --import-source on -k regex:arcv_stream_kernel -s 3 -c 1 \
   -o $OUT/${TAG}_k1_c4 -f python bench.py --profile --steps 1 --warmup 3 > $OUT/${TAG}_k1_c4.log 2>&1
 echo "k1 rc=$?"
-$NCU --set full --clock-control none --import-source on -k regex:arcv_compact_kernel -s 3 -c 1 \
-  -o $OUT/${TAG}_k2_c4 -f python bench.py --profile --steps 1 --warmup 3 > $OUT/${TAG}_k2_c4.log 2>&1
-echo "k2 rc=$?"
 $NCU --set full --clock-control none --import-source on -k regex:arcv_stream_kernel -s 3 -c 1 \
   -o $OUT/${TAG}_k1_c2a -f python -c "
 import sys; sys.path.insert(0, '.')
@@ -28,7 +25,7 @@ for _ in range(5): av.compare(o, r, 0.0, 1e-5, 1 << 20)
 torch.cuda.synchronize(); av.finalize()
 " > $OUT/${TAG}_k1_c2a.log 2>&1
 echo "k1 c2a rc=$?"
-for f in k1_c4 k2_c4 k1_c2a; do
+for f in k1_c4 k1_c2a; do
   $NCU -i $OUT/${TAG}_$f.ncu-rep --page raw --csv > $OUT/${TAG}_${f}_raw.csv 2>/dev/null
   $NCU -i $OUT/${TAG}_$f.ncu-rep --page details --csv > $OUT/${TAG}_${f}_details.csv 2>/dev/null
 done
