@@ -821,7 +821,7 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
         bulk_g2s(dst + kStageArrayBytes, reinterpret_cast<const void *>(ar), nbr, &sh.bar[st], policy);
     };
     // wait for tile `key` in stage st, write its entries from report rank excl
-    auto emit = [&](uint64_t key, uint64_t excl, int st, bool direct) {
+    auto emit = [&](uint64_t key, uint64_t excl, int st, bool direct, bool stamp = false) {
         const Seg &g = segs[key >> 40];
         StageInfo si;
         uintptr_t ao, ar;
@@ -829,16 +829,16 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
         plan_tile(g, key & kLtMask, si, ao, nbo, ar, nbr);
         mbar_wait(&sh.bar[st], phase[st]);
         phase[st] ^= 1u;
-        if (tid == 0) ARCV_STAMP(1, 4);
+        if (tid == 0 && stamp) ARCV_STAMP(1, 4);
         if (excl < g.max_report) {  // uniform
             if ((direct || (g.flags & kSegReportHost)) && tid == 0) sh.wrote = 1;
             const uint8_t *so = smem + (size_t)st * kStageBytes;
             const uint64_t mask = mask_any(so, so + kStageArrayBytes, si, tid, g);
-            if (tid == 0) ARCV_STAMP(1, 5);
+            if (tid == 0 && stamp) ARCV_STAMP(1, 5);
             compact_any(g, si, so, so + kStageArrayBytes, mask, excl | (direct ? kDirectBit : 0ull), sh.w, tid);
         }
         consumer_bar();  // stage `st` and sh.w are reused
-        if (tid == 0) ARCV_STAMP(1, 2);
+        if (tid == 0 && stamp) ARCV_STAMP(1, 2);
     };
 
     const uint32_t n_nz = *(volatile uint32_t *)p.nz_cnt;
@@ -847,6 +847,12 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
         // ------------------------------------------------------ pool path
         // arrive on the grid-barrier counter without waiting (host base += grid)
         if (tid == 0) atomicAdd(p.gbar, 1ull);
+#if defined(ARCV_TAIL_REPS)
+      // diagnostic: run the (idempotent) pool path again, stamps from the last run
+      for (int rep_ = 0; rep_ < ARCV_TAIL_REPS; ++rep_) {
+        consumer_bar();
+        if (tid == 0) ARCV_STAMP(1, 8);
+#endif
         const uint32_t n_own = n_nz > b ? (n_nz - b + G - 1) / G : 0u;
         if (tid == 0)
             for (uint32_t j = 0; j < n_own && j < 2; ++j) issue(__ldcg(p.nz_list + 2 * (b + j * G)), (int)j);
@@ -862,6 +868,9 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
             pk[u] = e.x;
             pc[u] = e.y;
         }
+#if defined(ARCV_TRACE) && ARCV_TRACE
+        if (tid == 0 && pk[0] != 1ull) ARCV_STAMP(1, 9);  // waits for the first pool load
+#endif
         for (uint32_t j0 = 0; j0 < n_own; j0 += 2) {
             const uint32_t m = n_own - j0 < 2u ? n_own - j0 : 2u;
             uint64_t key[2], pre[2] = {0, 0}, tot[2] = {0, 0};
@@ -904,11 +913,15 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
                 // a sparse region with a pinned host report: written over PCIe
                 // directly (the host then skips its D2H copy; same rule there)
                 const bool direct = g.report_alias && !(g.flags & kSegBaseFromAcc) && seg_tot <= kDirectDyn;
-                emit(key[q], base + r[q], st, direct);  // ends with a barrier: sh.red free again
+                emit(key[q], base + r[q], st, direct, j == 0);  // ends with a barrier: sh.red free again
+                if (tid == 0 && j == 1) ARCV_STAMP(1, 10);
                 if (tid == 0 && j + 2 < n_own) issue(__ldcg(p.nz_list + 2 * (b + (j + 2) * G)), st);
             }
         }
         if (tid == 0) ARCV_STAMP(1, 6);
+#if defined(ARCV_TAIL_REPS)
+      }
+#endif
     } else {
         // ------------------------------------------------------ group path
         for (uint32_t sgi = 0; sgi < p.n_segs; ++sgi) {
@@ -990,9 +1003,11 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
 #else
     const bool wrote_host = false;
 #endif
-    if (p.finalize)
-        finalize_launch(p, tid, kConsumerThreads, &sh.last, wrote_host, done_base,
-                        !(k1_published_if_empty && n_nz == 0));
+    if (p.finalize) {
+        const bool last = last_cta(p, tid, kConsumerThreads, &sh.last, wrote_host, done_base);
+        if (tid == 0) ARCV_STAMP(1, 11);
+        if (last && !(k1_published_if_empty && n_nz == 0)) publish(p, tid, kConsumerThreads);
+    }
     if (tid == 0) ARCV_STAMP(1, 7);
 }
 

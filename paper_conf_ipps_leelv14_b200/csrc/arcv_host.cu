@@ -123,7 +123,7 @@ constexpr uint64_t kDirectReportMax = 1 << 16;
 
 // Device alias of page-locked host memory (cudaMallocHost / cudaHostRegister /
 // torch pin_memory), or NULL.  Kernels write small results there directly.
-static void *pinned_device_alias(const void *p) {
+void *pinned_device_alias(const void *p) {
     cudaPointerAttributes a;
     if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
         cudaGetLastError();

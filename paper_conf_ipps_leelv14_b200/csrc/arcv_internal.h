@@ -89,6 +89,7 @@ extern Ctx *g_ctx;
 void set_error(const char *fmt, ...);
 int cuda_fail(cudaError_t e, const char *what);
 PtrKind classify(const void *p, int device);
+void *pinned_device_alias(const void *p);  // device alias of pinned host memory, else nullptr
 int validate_region(const void *out, const void *ref, uint64_t n, int dtype, double abs_tol, double rel_tol,
                     uint64_t max_report, const arc_verify_result_t *res);
 int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_t n_acc, bool finalize);

@@ -63,8 +63,10 @@ struct PeerParams {
     unsigned long long s;           // collective sequence number = flag value
     uint64_t n_local, max_report, cap;
     const Acc *mirror;              // local summary (written by the local compare)
-    arc_mismatch_t *dst;            // global report target (device or pinned alias), or nullptr
-    int dst_host;                   // dst is mapped host memory (system-scope fences)
+    arc_mismatch_t *dst;            // global report target (device memory or HBM staging), or nullptr
+    arc_mismatch_t *dst_alias;      // device alias of the caller's pinned host report, or nullptr:
+                                    // used instead of dst when the global report has <= kDirectDyn
+                                    // entries (the host then skips its D2H copy; same rule there)
     arc_shard_header_t *out;        // mapped host: [0] global header, [1].n = status (1 = timeout)
     unsigned long long *done;       // monotonic finished-block counter
     unsigned long long done_base;
@@ -80,6 +82,9 @@ __device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long
     asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
     return v;
 }
+// message-passing fences (no fence.sc needed; see arcv_device.cuh fence_gpu/fence_sys)
+__device__ __forceinline__ void peer_fence_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+__device__ __forceinline__ void peer_fence_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
 __device__ __forceinline__ unsigned long long ld_volatile(const unsigned long long *p) {
     return *reinterpret_cast<const volatile unsigned long long *>(p);
 }
@@ -106,7 +111,7 @@ __global__ void __launch_bounds__(256) arcv_peer_kernel(const __grid_constant__ 
         h[1] = q.mirror->count;
         h[2] = q.mirror->max_abs_bits;
         h[3] = q.mirror->max_rel_bits;
-        __threadfence_system();  // header + the local report (previous kernels) before the flags
+        peer_fence_sys();  // header + the local report (previous kernels) before the flags
         for (int r = 0; r < q.p; ++r) st_release_sys(flag_slot(q.win[r], q.par, q.rank), q.s);
     }
     // 2. wait for every rank's flag in the own window
@@ -145,6 +150,7 @@ __global__ void __launch_bounds__(256) arcv_peer_kernel(const __grid_constant__ 
         }
         __syncthreads();
         total = q.dst ? cum[q.p] : 0;
+        arc_mismatch_t *const dst = (q.dst_alias && total <= kDirectDyn) ? q.dst_alias : q.dst;
         for (uint64_t gi = (uint64_t)blockIdx.x * blockDim.x + tid; gi < total;
              gi += (uint64_t)gridDim.x * blockDim.x) {
             int lo = 0, hi = q.p;  // last r with cum[r] <= gi
@@ -159,23 +165,24 @@ __global__ void __launch_bounds__(256) arcv_peer_kernel(const __grid_constant__ 
             e.index = ld_volatile(src) + plan[lo].index_offset;
             e.out_bits = ld_volatile(src + 1);
             e.ref_bits = ld_volatile(src + 2);
-            q.dst[plan[lo].prefix + j] = e;
+            dst[plan[lo].prefix + j] = e;
         }
     }
     // 4. completion: the last block publishes the global header, then the word
     __syncthreads();
     if (tid == 0) {
         if (!ok) q.out[1].n = 1;  // status: timed out
-        if (q.dst_host || !ok) __threadfence_system();
-        else __threadfence();
+        // gpu-scope release: the last block's system fence below is cumulative
+        // (entries written to a pinned host report included)
+        peer_fence_gpu();
         const unsigned long long prev = atomicAdd(q.done, 1ull);
         s_last = (prev - q.done_base) == (unsigned long long)(gridDim.x - 1);
     }
     __syncthreads();
     if (s_last && tid == 0) {
-        __threadfence();
+        peer_fence_gpu();
         if (ok) q.out[0] = glob;
-        __threadfence_system();
+        peer_fence_sys();
         *(volatile unsigned long long *)q.done_flag = q.seq;
     }
 }
@@ -243,7 +250,8 @@ int peer_compare(Ctx &c, const arc_verify_region_t &r, arc_verify_result_t *resu
     q.cap = c.win_cap;
     q.mirror = c.mirror;
     q.dst = dst;
-    q.dst_host = 0;
+    // a sparse global report goes straight into a pinned caller buffer
+    q.dst_alias = host_report ? static_cast<arc_mismatch_t *>(pinned_device_alias(result->report)) : nullptr;
     q.out = c.peer_out_dev;
     q.done = c.counters + 5;
     q.done_base = c.peer_done_base;
@@ -271,7 +279,7 @@ int peer_compare(Ctx &c, const arc_verify_region_t &r, arc_verify_result_t *resu
         return ARC_E_CUDA;
     }
     fill_result(c.peer_out_host[0], r.max_report, result);
-    if (host_report && result->n_reported) {
+    if (host_report && result->n_reported && !(q.dst_alias && result->n_reported <= kDirectDyn)) {
         CK(cudaMemcpyAsync(result->report, dst, result->n_reported * sizeof(arc_mismatch_t), cudaMemcpyDeviceToHost,
                            c.stream));
         CK(cudaStreamSynchronize(c.stream));

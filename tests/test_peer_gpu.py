@@ -67,6 +67,10 @@ def _worker(rank, world, port, q):
 
         torch.cuda.set_device(0)
         assert av.init_distributed(transport="peer", max_report_cap=1 << 14) == "peer"
+        # report buffers: pageable (HBM staging + D2H), pinned (a sparse global report is
+        # written by the exchange kernel straight over PCIe), device memory
+        pinned = torch.empty(24 << 14, dtype=torch.uint8, pin_memory=True).numpy().view(av.REPORT_DTYPE)
+        dev_rep = torch.empty(24 << 14, dtype=torch.uint8, device="cuda")
         for name, mk, (at, rt), dt in _cases():
             reg = mk()
             for kind in ("even", "ragged", "empty0"):
@@ -74,11 +78,15 @@ def _worker(rank, world, port, q):
                 a, b = cuts[rank], cuts[rank + 1]
                 o, r = reg.slice(a, b - a, device="cuda")
                 for mr in (0, 7, 100, 1 << 14):
-                    for rep in range(2):  # consecutive calls alternate the window parity
-                        g = av.compare(o, r, at, rt, mr)
+                    for rep in range(3):  # consecutive calls alternate the window parity
+                        buf = (None, pinned, dev_rep)[rep]
+                        g = av.compare(o, r, at, rt, mr, report=buf)
+                        entries = g.report
+                        if isinstance(entries, torch.Tensor):
+                            entries = entries.cpu().numpy().view(av.REPORT_DTYPE)[: g.n_reported]
                         out.append(((name, kind, mr, rep), (g.n, g.n_mismatch, _bits(g.max_abs_err),
                                                             _bits(g.max_rel_err), g.n_reported,
-                                                            np.array(g.report).tobytes())))
+                                                            np.array(entries[: g.n_reported]).tobytes())))
         # a report larger than the window with no NCCL communicator: refused, not wrong
         try:
             av.compare(o, r, 0, 0, (1 << 14) + 1)
@@ -128,7 +136,7 @@ def test_peer_exchange_matches_unsharded_oracle(world):
             want = (e.n, e.n_mismatch, _bits(e.max_abs_err), _bits(e.max_rel_err), e.n_reported,
                     np.ascontiguousarray(e.report).tobytes())
             for kind in ("even", "ragged", "empty0"):
-                for rep in range(2):
+                for rep in range(3):
                     got = res[0][(name, kind, mr, rep)]
                     assert got[:5] == want[:5], (name, kind, mr, rep, got[:5], want[:5])
                     assert got[5] == want[5], (name, kind, mr, rep)

@@ -24,8 +24,9 @@ REP = torch.empty(24 * (1 << 20), dtype=torch.uint8, pin_memory=True).numpy().vi
 P, U64, I, D = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int, ctypes.c_double
 lib.arc_verify_compare.argtypes = [P, P, U64, I, D, D, U64, ctypes.POINTER(av.arc_verify_result_t)]
 K1 = ["start", "loop end", "flush end", "exit"]
-K2 = ["entry / barrier arrive", "after wait", "last tile emitted", "1st prefixes", "last tile landed",
-      "last tile masked", "pool loop end", "exit", "last rep start (TAIL_REPS)"]
+K2 = ["entry / barrier arrive", "after wait", "tile 0 emitted", "prefixes reduced", "tile 0 landed",
+      "tile 0 masked", "pool loop end", "exit", "last rep start (TAIL_REPS)", "pool loaded", "tile 1 emitted",
+      "after last_cta (fence+atomic+bar)"]
 
 
 def run(name, o, r, at, rt, mr):
