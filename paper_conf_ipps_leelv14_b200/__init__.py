@@ -519,6 +519,59 @@ def prepare(out, ref, abs_tol: float = 0.0, rel_tol: float = 0.0, max_report: in
     return Prepared(out, ref, abs_tol, rel_tol, max_report, report, n, min_value, bounds)
 
 
+class PreparedBatch:
+    """``pb = prepare_batch(regions)``: arc_verify_batch with the region table,
+    result structs and report buffers built once; each ``pb()`` is one C call
+    (one grid over every region).  Tensors must stay alive and in place."""
+
+    __slots__ = ("_regs", "_res", "_reps", "_n", "_keep")
+
+    def __init__(self, regions, report_buffers=None):
+        regions = list(regions)
+        R = len(regions)
+        self._n = R
+        self._regs = (arc_verify_region_t * R)()
+        self._res = (arc_verify_result_t * R)()
+        self._reps, keep = [], []
+        for k, reg in enumerate(regions):
+            out, ref, at, rt, mr = reg[:5]
+            name = reg[5] if len(reg) > 5 else None
+            n = out.numel()
+            if ref.numel() != n or out.dtype != ref.dtype:
+                raise ValueError(f"region {k}: size/dtype mismatch")
+            if n and not (out.is_contiguous() and ref.is_contiguous()):
+                raise ValueError(f"region {k}: tensors must be contiguous")
+            if report_buffers is not None and report_buffers[k] is not None:
+                arr = report_buffers[k]
+                ptr = arr.ctypes.data if isinstance(arr, np.ndarray) else arr.data_ptr()
+            else:
+                arr, ptr = _report_buffer(min(int(mr), n))
+            nm = name.encode() if name else None
+            ck = reg[6] if len(reg) > 6 else None
+            self._regs[k] = arc_verify_region_t(out.data_ptr() if n else None, ref.data_ptr() if n else None, n,
+                                                dtype_code(out), float(at), float(rt), int(mr), nm,
+                                                ctypes.pointer(ck) if ck is not None else None)
+            self._res[k].report = ptr if mr > 0 else None
+            self._reps.append(arr)
+            keep.append((out, ref, nm, ck))
+        self._keep = keep
+
+    def __call__(self) -> list[Result]:
+        _check(_lib.arc_verify_batch(self._regs, self._n, self._res), "arc_verify_batch")
+        outs = []
+        for k in range(self._n):
+            r = self._res[k]
+            nr = int(r.n_reported)
+            rep = self._reps[k][:nr] if isinstance(self._reps[k], np.ndarray) else self._reps[k]
+            outs.append(Result(int(r.n), int(r.n_mismatch), float(r.max_abs_err), float(r.max_rel_err), nr, rep))
+        return outs
+
+
+def prepare_batch(regions, report_buffers=None) -> PreparedBatch:
+    """Validate and marshal a batch once (see PreparedBatch)."""
+    return PreparedBatch(regions, report_buffers)
+
+
 def batch(regions, options: Optional[str] = None, select: bool = False) -> list[Result]:
     """regions: iterable of (out, ref, abs_tol, rel_tol, max_report[, name[, check]]) with torch
     tensors; ``check`` is an arc_verify_check_t (see make_check) or None."""

@@ -820,9 +820,15 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
         bulk_g2s(dst, reinterpret_cast<const void *>(ao), nbo, &sh.bar[st], policy);
         bulk_g2s(dst + kStageArrayBytes, reinterpret_cast<const void *>(ar), nbr, &sh.bar[st], policy);
     };
-    // wait for tile `key` in stage st, write its entries from report rank excl
-    auto emit = [&](uint64_t key, uint64_t excl, int st, bool direct, bool stamp = false) {
+    // wait for tile `key` in stage st, write its entries from report rank excl.
+    // A region with a report_alias (pinned host memory, the caller's or the
+    // library's staging for a pageable buffer) and at most kDirectDyn
+    // mismatches in total -- K1's final count; the host applies the same rule
+    // to n_mismatch -- gets its entries written there directly over PCIe.
+    auto emit = [&](uint64_t key, uint64_t excl, int st, bool stamp = false) {
         const Seg &g = segs[key >> 40];
+        const bool direct = g.report_alias && !(g.flags & kSegBaseFromAcc) &&
+                            __ldcg(&p.acc[g.acc_slot].count) <= kDirectDyn;
         StageInfo si;
         uintptr_t ao, ar;
         uint32_t nbo, nbr;
@@ -854,8 +860,12 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
         if (tid == 0) ARCV_STAMP(1, 8);
 #endif
         const uint32_t n_own = n_nz > b ? (n_nz - b + G - 1) / G : 0u;
-        if (tid == 0)
-            for (uint32_t j = 0; j < n_own && j < 2; ++j) issue(__ldcg(p.nz_list + 2 * (b + j * G)), (int)j);
+        if (tid == 0 && n_own > 0) {  // both key loads in flight before the first issue
+            const uint64_t k0 = __ldcg(p.nz_list + 2 * b);
+            const uint64_t k1 = n_own > 1 ? __ldcg(p.nz_list + 2 * (b + G)) : 0ull;
+            issue(k0, 0);
+            if (n_own > 1) issue(k1, 1);
+        }
         // the whole pool in registers, all loads in flight at once: entry
         // tid + u * 256 = {seg << 40 | tile, count}; absent entries never match
         constexpr int kPer = kPoolCap / kConsumerThreads;
@@ -910,10 +920,7 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
                 uint64_t base = 0;
                 if (g.flags & kSegBaseFromAcc) base = __ldcg(&p.acc[g.acc_slot].count) - seg_tot;
                 if (tid == 0) p.tile_cnt[g.slot_begin + (key[q] & kLtMask)] = 0u;  // clean for the next call
-                // a sparse region with a pinned host report: written over PCIe
-                // directly (the host then skips its D2H copy; same rule there)
-                const bool direct = g.report_alias && !(g.flags & kSegBaseFromAcc) && seg_tot <= kDirectDyn;
-                emit(key[q], base + r[q], st, direct, j == 0);  // ends with a barrier: sh.red free again
+                emit(key[q], base + r[q], st, j == 0);  // ends with a barrier: sh.red free again
                 if (tid == 0 && j == 1) ARCV_STAMP(1, 10);
                 if (tid == 0 && j + 2 < n_own) issue(__ldcg(p.nz_list + 2 * (b + (j + 2) * G)), st);
             }
@@ -988,7 +995,7 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
             if (j + 1 < mine && tid == 0) issue(__ldcg(p.active + 2 * (b + (j + 1) * G)), st ^ 1);  // prefetch
             const uint64_t key = __ldcg(p.active + 2 * (b + j * G));
             const uint64_t excl = __ldcg(p.active + 2 * (b + j * G) + 1);
-            emit(key, excl, st, false);
+            emit(key, excl, st);
         }
     }
     // Report entries in pinned host memory need no system-scope fence here:

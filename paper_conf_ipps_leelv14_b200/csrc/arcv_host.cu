@@ -245,11 +245,16 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
     } else {
         st = grow_device(&c.seg_dev, &c.seg_dev_cap, n_segs, false, c.stream);
         if (st) return st;
+        // seg_host may still feed the previous table copy: wait for that copy
+        // only (an event after it), not for the whole stream
+        if (c.seg_copy_pending) CK(cudaEventSynchronize(c.ev_seg));
+        c.seg_copy_pending = false;
         st = grow_pinned(&c.seg_host, &c.seg_host_cap, n_segs);
         if (st) return st;
-        CK(cudaStreamSynchronize(c.stream));  // seg_host may still feed an earlier copy
         memcpy(c.seg_host, segs, n_segs * sizeof(Seg));
         CK(cudaMemcpyAsync(c.seg_dev, c.seg_host, n_segs * sizeof(Seg), cudaMemcpyHostToDevice, c.stream));
+        CK(cudaEventRecord(c.ev_seg, c.stream));
+        c.seg_copy_pending = true;
         p.segs = c.seg_dev;
     }
     p.n_segs = n_segs;
@@ -476,11 +481,13 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
         arc_mismatch_t *dreport;  // device target
         arc_mismatch_t *alias;    // device alias of a pinned host report (sparse: written directly)
         bool host_report;
-        uint64_t stage_off;
+        bool pageable;            // host report in pageable memory: sparse entries land in the
+                                  // library's pinned staging (pin_off), then one host memcpy
+        uint64_t stage_off, pin_off;
         uint64_t tiles, slot_base;
     };
     std::vector<Plan> plan(R);
-    uint64_t tile_slots = 0, stage_entries = 0;
+    uint64_t tile_slots = 0, stage_entries = 0, pin_entries = 0;
     for (size_t k = 0; k < R; ++k) {
         const arc_verify_region_t &r = regs[k];
         int st = validate_region(r.out, r.ref, r.n, r.dtype, r.abs_tol, r.rel_tol, r.max_report, &results[k]);
@@ -504,6 +511,7 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
         tile_slots += pl.tiles;
         const uint64_t cap = std::min<uint64_t>(r.max_report, r.n);
         pl.host_report = false;
+        pl.pageable = false;
         pl.dreport = nullptr;
         pl.alias = nullptr;
         if (cap > 0) {
@@ -517,7 +525,14 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
                 pl.host_report = true;
                 pl.stage_off = stage_entries;
                 stage_entries += cap;
-                if (!pl.stream) pl.alias = static_cast<arc_mismatch_t *>(pinned_device_alias(results[k].report));
+                if (!pl.stream) {
+                    pl.alias = static_cast<arc_mismatch_t *>(pinned_device_alias(results[k].report));
+                    if (!pl.alias) {  // pageable: the sparse case goes through pinned staging
+                        pl.pageable = true;
+                        pl.pin_off = pin_entries;
+                        pin_entries += std::min<uint64_t>(cap, kDirectDyn);
+                    }
+                }
             }
         }
     }
@@ -527,6 +542,26 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
         st = grow_device(&c.report_stage, &c.report_stage_cap, stage_entries, false, c.stream);
         if (st) return st;
     }
+    if (pin_entries > c.report_pin_cap) {  // mapped pinned staging for sparse pageable reports
+        if (c.report_pin) {
+            CK(cudaStreamSynchronize(c.stream));
+            CK(cudaFreeHost(c.report_pin));
+        }
+        c.report_pin = nullptr;
+        c.report_pin_cap = 0;
+        const size_t cap = std::max<size_t>(pin_entries, 2 * kDirectDyn);
+        cudaError_t e = cudaHostAlloc(reinterpret_cast<void **>(&c.report_pin), cap * sizeof(arc_mismatch_t),
+                                      cudaHostAllocMapped);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            set_error("cudaHostAlloc(report staging) failed: %s", cudaGetErrorString(e));
+            return ARC_E_NOMEM;
+        }
+        CK(cudaHostGetDevicePointer(reinterpret_cast<void **>(&c.report_pin_dev), c.report_pin, 0));
+        c.report_pin_cap = cap;
+    }
+    for (size_t k = 0; k < R; ++k)
+        if (plan[k].pageable) plan[k].alias = c.report_pin_dev + plan[k].pin_off;
     for (size_t k = 0; k < R; ++k)
         if (plan[k].host_report) plan[k].dreport = c.report_stage + plan[k].stage_off;
 
@@ -588,7 +623,12 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
         bool any = false;
         for (size_t k = 0; k < R; ++k) {
             if (!plan[k].host_report || results[k].n_reported == 0) continue;
-            if (plan[k].alias && results[k].n_mismatch <= kDirectDyn) continue;  // K2 wrote it directly
+            if (plan[k].alias && results[k].n_mismatch <= kDirectDyn) {  // the kernel wrote it directly
+                if (plan[k].pageable)
+                    memcpy(results[k].report, c.report_pin + plan[k].pin_off,
+                           results[k].n_reported * sizeof(arc_mismatch_t));
+                continue;
+            }
             CK(cudaMemcpyAsync(results[k].report, plan[k].dreport, results[k].n_reported * sizeof(arc_mismatch_t),
                                cudaMemcpyDeviceToHost, c.stream));
             any = true;
@@ -661,6 +701,7 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
         CK(cudaEventCreateWithFlags(&c->ev_copy[b], cudaEventDisableTiming));
         CK(cudaEventCreateWithFlags(&c->ev_free[b], cudaEventDisableTiming));
     }
+    CK(cudaEventCreateWithFlags(&c->ev_seg, cudaEventDisableTiming));
     for (int i = 0; i < Ctx::kMaxEv; ++i) {
         CK(cudaEventCreate(&c->ev[i][0]));
         CK(cudaEventCreate(&c->ev[i][1]));
@@ -744,7 +785,9 @@ int arc_verify_finalize(void) {
     if (c->result_host) cudaFreeHost(c->result_host);  // result_dev is its device alias
     if (c->flag_host) cudaFreeHost(c->flag_host);
     if (c->seg_host) cudaFreeHost(c->seg_host);
+    if (c->report_pin) cudaFreeHost(c->report_pin);  // report_pin_dev is its device alias
     if (c->hdr_host) cudaFreeHost(c->hdr_host);
+    if (c->ev_seg) cudaEventDestroy(c->ev_seg);
     for (int b = 0; b < Ctx::kNBuf; ++b) {
         cudaFree(c->chunk_buf[b][0]);
         cudaFree(c->chunk_buf[b][1]);

@@ -49,7 +49,12 @@ struct Ctx {
     Acc *result_dev = nullptr;                                       // its device alias
     Seg *seg_dev = nullptr;            size_t seg_dev_cap = 0;
     Seg *seg_host = nullptr;           size_t seg_host_cap = 0;
+    cudaEvent_t ev_seg = nullptr;      // after the last segment-table copy
+    bool seg_copy_pending = false;
     arc_mismatch_t *report_stage = nullptr; size_t report_stage_cap = 0;
+    arc_mismatch_t *report_pin = nullptr;      // mapped pinned staging (sparse pageable reports)
+    arc_mismatch_t *report_pin_dev = nullptr;  // its device alias
+    size_t report_pin_cap = 0;
 
     void *chunk_buf[kNBuf][2] = {{nullptr, nullptr}, {nullptr, nullptr}};
     cudaEvent_t ev_copy[kNBuf] = {}, ev_free[kNBuf] = {};

@@ -14,7 +14,7 @@ constexpr int kConsumerWarps = 8;
 constexpr int kConsumerThreads = kConsumerWarps * 32;
 constexpr int kThreads = kConsumerThreads + 32;     // + producer warp
 constexpr int kVecPerThread = kTileBytes / 16 / kConsumerThreads;  // 4
-constexpr int kMaxInlineSegs = 8;
+constexpr int kMaxInlineSegs = 16;                 // regions passed as kernel parameters (C3: 12)
 constexpr int kGroupTiles = 256;                    // tiles per group counter
 constexpr int kPoolCap = 2048;                      // K2 pool path: max listed nonzero tiles
 constexpr uint64_t kDirectDyn = 4096;               // sparse reports: K2 writes a pinned host report directly
@@ -90,6 +90,8 @@ struct Params {
     uint32_t flags;
     Seg inline_segs[kMaxInlineSegs];
 };
+
+static_assert(sizeof(Params) <= 4096, "kernel parameters stay within the classic 4 KB limit");
 
 struct StageInfo {
     uint64_t tile;        // launch-local tile, ~0 = no more work

@@ -205,6 +205,11 @@ def test_c3_batch_matches_oracle_and_singles(av, orc):
         assert list(g.report["index"]) == reg.planted()
         single = av.compare(o, r, reg.abs_tol, reg.rel_tol, reg.max_report)
         assert_same(single, exp, reg.name + " single")
+    # the prepared batch (table built once), called repeatedly, gives the same results
+    pb = av.prepare_batch([(o, r, reg.abs_tol, reg.rel_tol, reg.max_report, reg.name) for reg, o, r in data])
+    for _ in range(3):
+        for g, h in zip(pb(), res):
+            assert_same(g, h, "prepared batch")
 
 
 def test_c3_batch_misaligned_packing(av, orc):
@@ -229,7 +234,7 @@ def test_c3_batch_misaligned_packing(av, orc):
 
 
 def test_batch_many_regions_table_path(av, orc):
-    """> 8 segments go through the device descriptor table; include empty regions."""
+    """> 16 segments go through the device descriptor table; include empty regions."""
     items, exps = [], []
     for k in range(37):
         dt = ["f32", "f64", "i32", "i64", "u8"][k % 5]
@@ -239,6 +244,42 @@ def test_batch_many_regions_table_path(av, orc):
         exps.append(orc.compare(o.cpu().numpy(), r.cpu().numpy(), dt, 1e-6, 1e-5, [0, 3, 1000][k % 3]))
     for g, e in zip(av.batch(items), exps):
         assert_same(g, e)
+    # the pinned descriptor table is reused call after call (event-ordered, no stream sync)
+    pb = av.prepare_batch(items)
+    half = av.prepare_batch(items[::2])
+    for _ in range(3):
+        for g, e in zip(pb(), exps):
+            assert_same(g, e, "prepared")
+        for g, e in zip(half(), exps[::2]):
+            assert_same(g, e, "prepared half")
+
+
+@pytest.mark.parametrize("buf", ["pinned_large", "pageable"])
+def test_batch_sparse_region_next_to_dense(av, orc, buf):
+    """A sparse region (10 mismatches) batched with a dense one that overflows the pool
+    (> 2048 nonzero tiles -> group path): the sparse region's entries take the direct
+    route (pinned caller buffer, or the library's pinned staging for a pageable one) on
+    both report paths, and the host applies the same rule."""
+    oa, ra = random_pair("f32", 300_000, seed=71, rate=0.0)
+    idx = torch.tensor([5, 77, 4096, 9000, 123456, 200001, 250000, 299990, 299998, 299999])
+    oa[idx.cuda()] += 1.0
+    ob, rb = synth.C5(1 << 24).slice(device="cuda")  # 4096 nonzero tiles
+    cap = 100_000  # > the 2^16 small-pinned limit: the sparse rule decides
+    if buf == "pinned_large":
+        rep_a = torch.empty(24 * cap, dtype=torch.uint8, pin_memory=True).numpy().view(av.REPORT_DTYPE)
+    else:
+        rep_a = np.zeros(cap, dtype=av.REPORT_DTYPE)
+    pb = av.prepare_batch([(oa, ra, 1e-6, 1e-5, cap), (ob, rb, 0, 0, 5000)], report_buffers=[rep_a, None])
+    ea = orc.compare(oa.cpu().numpy(), ra.cpu().numpy(), "f32", 1e-6, 1e-5, cap)
+    eb = orc.compare(ob.cpu().numpy(), rb.cpu().numpy(), "i32", 0, 0, 5000)
+    for _ in range(2):
+        rep_a[:] = np.zeros(1, dtype=av.REPORT_DTYPE)  # stale-free check
+        ga, gb = pb()
+        assert_same(ga, ea, f"sparse {buf}")
+        assert_same(gb, eb, "dense")
+    # and the same region alone (pool path)
+    g = av.compare(oa, ra, 1e-6, 1e-5, cap, report=rep_a)
+    assert_same(g, ea, f"alone {buf}")
 
 
 # ----------------------------------------------------------- host inputs

@@ -82,8 +82,9 @@ def main():
     data = [rg.slice(device="cuda") for rg in regs]
     nb = sum(2 * o.numel() * o.element_size() for o, _ in data)
     tup = [(o, r, rg.abs_tol, rg.rel_tol, rg.max_report, rg.name) for rg, (o, r) in zip(regs, data)]
-    b = av.batch(tup)
-    line("C3 batch (1 call, 12 regions)", nb, *timed(lambda: av.batch(tup), nb, True), 0.0,
+    pb = av.prepare_batch(tup)
+    b = pb()
+    line("C3 batch (1 call, 12 regions)", nb, *timed(pb, nb, True), 0.0,
          f"mism={sum(x.n_mismatch for x in b)}")
     singles = [av.prepare(o, r, rg.abs_tol, rg.rel_tol, rg.max_report) for rg, (o, r) in zip(regs, data)]
 

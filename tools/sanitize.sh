@@ -7,3 +7,9 @@ for tool in memcheck racecheck synccheck initcheck; do
     > gpurun_out/san_$tool.log 2>&1
   echo "$tool rc=$?"; tail -1 gpurun_out/san_$tool.log
 done
+# the separate report kernel (K2) instead of K1's fused tail
+for tool in racecheck synccheck; do
+  ARCV_FUSED=0 /usr/local/cuda/bin/compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize_workload.py \
+    > gpurun_out/san_${tool}_k2.log 2>&1
+  echo "$tool (ARCV_FUSED=0) rc=$?"; tail -1 gpurun_out/san_${tool}_k2.log
+done
