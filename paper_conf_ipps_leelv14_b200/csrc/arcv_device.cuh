@@ -1,6 +1,6 @@
 // arcv_device.cuh -- sm_100a kernels of the kernel-verification comparison.
 //
-// Two kernels per verification call:
+// One kernel per verification call:
 //
 //  K1 arcv_stream_kernel  -- a2-a4 (+ the counting half of a5).  A persistent
 //     grid streams both arrays of every segment through a cp.async.bulk (TMA
@@ -10,11 +10,14 @@
 //     it also records per-tile and per-group (256 tiles) mismatch counts with
 //     warp-level atomics -- no block barrier, no inter-CTA waiting in the
 //     streaming loop.
-//  K2 arcv_compact_kernel -- a5.  Scans the group and tile counts (tiny), and
-//     re-reads ONLY the tiles whose mismatches fall among the first max_report
-//     (exclusive prefix < max_report), writing their entries in ascending index
-//     order.  Sparse mismatches cost one extra tile read each; dense ones stop
-//     at max_report.  The last CTA to finish publishes the per-region summary.
+//  report_phase -- a5, run by K1's consumer warps after a grid barrier when a
+//     region wants a report (K1 is then a cooperative launch), or as its own
+//     kernel K2 arcv_compact_kernel (fewer than 3 stages, or ARCV_FUSED=0).
+//     Scans the group and tile counts (tiny), and re-reads ONLY the tiles whose
+//     mismatches fall among the first max_report (exclusive prefix <
+//     max_report), writing their entries in ascending index order.  Sparse
+//     mismatches cost one extra tile read each; dense ones stop at max_report.
+//     The last CTA to finish publishes the per-region summary.
 //
 // Block of K1 = 1 producer warp (one lane issues bulk copies; tile tickets come
 // from a global atomic so the grid is load-balanced) + 8 consumer warps.  A tile
@@ -310,7 +313,7 @@ __device__ __forceinline__ void seed_bounds(const uint8_t *so, const uint8_t *sr
 }
 
 // Evaluate this thread's share of one tile; returns its number of mismatches
-// (K1 needs only counts; K2 re-derives the positions of the tiles it reports).
+// (K1 needs only counts; the report phase re-derives the positions of the tiles it reports).
 // Thread element order: bit k*EPV + j <-> tile element (k*256 + ctid)*EPV + j.
 // Floats: a fast pass over all elements with the exact pre-filter, then the
 // fp64 rule only for the (rare) flagged elements, re-read from the still-held
@@ -558,7 +561,7 @@ __device__ __forceinline__ void flush_acc(Acc *acc_base, uint32_t slot, uint32_t
 // clears them for the next call (monotonic done counter, host-tracked base).
 // It then stores the call's sequence number to a mapped host word, which the
 // host polls instead of a stream synchronise; system-scope fences order report
-// entries written to pinned host memory (K2, `wrote_host`) and the results
+// entries written to pinned host memory (report phase, `wrote_host`) and the results
 // before that word.
 __device__ __forceinline__ bool last_cta(const Params &p, int tid, int nthreads, int *s_last, bool wrote_host,
                                          unsigned long long base) {
@@ -602,7 +605,7 @@ __device__ __forceinline__ void finalize_launch(const Params &p, int tid, int nt
     if (last_cta(p, tid, nthreads, s_last, wrote_host, base) && do_publish) publish(p, tid, nthreads);
 }
 
-// --------------------------------------------------------------- K2 helpers
+// ------------------------------------------------------ report-phase helpers
 // Exclusive scan over the 256 consumer threads (named barrier 1; `tid` = the
 // consumer index, so K1's consumer warps can run it too) of a u64; returns the
 // exclusive prefix, writes the block total to *total.
@@ -664,8 +667,8 @@ __device__ __noinline__ void compact_tile(const Seg &g, const StageInfo &si, con
     }
 }
 
-// ------------------------------------------------------------- K2: mask only
-// K2 needs only the mismatch decision of each element of a re-read tile (the
+// ----------------------------------------------------- report phase: mask only
+// The report phase needs only the mismatch decision of each element of a re-read tile (the
 // maxima were taken by K1).  A compact, non-unrolled loop of the plain rule:
 // small code matters here because every CTA executes it cold, once.
 // The decision is the same rule K1 applies (its fast path only ever proves
@@ -728,14 +731,14 @@ __device__ __forceinline__ uint64_t mask_any(const uint8_t *so, const uint8_t *s
 #undef ARCV_MASK
 }
 
-// ---------------------------------------------------------------- K2: compact
+// ------------------------------------------------------- report phase: compact
 __device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long long *p) {
     unsigned long long v;
     asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
     return v;
 }
 
-// Software grid barrier (K2 is launched cooperatively, so all CTAs are
+// Software grid barrier (K1-with-report and K2 are cooperative launches, so all CTAs are
 // co-resident).  Monotonic counter; the host tracks each launch's base.
 // `tid` = consumer index; the 256 consumer threads synchronise on barrier 1.
 __device__ __forceinline__ void grid_barrier(unsigned long long *ctr, unsigned long long base, int tid) {
@@ -1122,7 +1125,7 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
         const uint32_t cnt = (p.flags & kFlagProbe) ? 0u : eval_any(so, so + kStageArrayBytes, si, ctid, g, acc);
         acc.count += cnt;
         if (g.max_report != 0) {
-            // Per-tile count for K2: warps fold their counts into the stage's
+            // Per-tile count for the report phase: warps fold their counts into the stage's
             // shared word (arrivals << 24 | count); the last warp publishes the
             // tile (2 global atomics per tile with mismatches, none otherwise)
             // and clears the word before the stage can be reused.
@@ -1136,7 +1139,7 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
                         const uint64_t lt = si.tile - g.tile_begin;
                         atomicAdd(p.tile_cnt + g.slot_begin + lt, tc);
                         atomicAdd(p.group_cnt + g.group_begin + lt / kGroupTiles, tc);
-                        // short list of nonzero tiles for K2's pool path (checked
+                        // short list of nonzero tiles for the pool path (checked
                         // before the atomic so a dense call stops touching it)
                         if (*(volatile uint32_t *)p.nz_cnt < (uint32_t)kPoolCap) {
                             const uint32_t k = atomicAdd(p.nz_cnt, 1u);
@@ -1153,7 +1156,7 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty_bar[s]);  // stage may be refilled now
     }
-    // K2 (programmatic dependent launch) may be scheduled from here on; it
+    // A dependent launch (exchange kernel or K2, PDL) may be scheduled from here on; it
     // waits for this grid's completion before reading anything it wrote.
     if (ctid == 0) ARCV_STAMP(0, 1);
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
@@ -1176,9 +1179,9 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
             return;
         }
     }
-    // The last CTA publishes at once unless K2 has report entries to write: with
-    // no mismatch in any reporting region (the common "verified clean" case)
-    // the host wakes here while K2 -- then a no-op -- runs in the background.
+    // Unfused (K2 follows): the last CTA publishes at once unless K2 has report
+    // entries to write: with no mismatch in any reporting region the host wakes
+    // here while K2 -- then a no-op -- runs in the background.
     if ((p.finalize || p.k2) && last_cta(p, ctid, kConsumerThreads, &s_last, false, p.done_base)) {
         fence_gpu();
         if (p.finalize && (!p.k2 || *(volatile uint32_t *)p.nz_cnt == 0u)) publish(p, ctid, kConsumerThreads);

@@ -208,7 +208,7 @@ static Seg make_seg(const void *out, const void *ref, uint64_t n, uint32_t dtype
 }
 
 // ------------------------------------------------------------------ launch
-// One K1 (+ K2 when any segment wants a report) over `segs`.  Fills each seg's
+// One K1 (its report phase fused, or + K2) over `segs`.  Fills each seg's
 // tile_begin / group_begin.  Accumulator slots [acc_lo, acc_lo + n_acc) are
 // published to the result slots when `finalize`.
 int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_t n_acc, bool finalize) {
@@ -279,7 +279,7 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
     p.gbar_base = c.gbar_base;
     p.acc = c.acc + acc_lo;
     p.result = c.result_dev + acc_lo;
-    p.finalize = finalize ? 1 : 0;  // K1 publishes unless K2 has report entries to write
+    p.finalize = finalize ? 1 : 0;  // the launch publishes the result slots
     p.flags = (uint32_t)c.flags;
     // ARCV_FLAGS bit 3 (diagnostic): stream sync; deferred (peer) calls wake on the exchange kernel
     p.done_flag = ((c.flags & 8) || c.defer_wait) ? nullptr : c.flag_dev;
@@ -520,7 +520,7 @@ int run_local(Ctx &c, const arc_verify_region_t *regs, size_t R, arc_verify_resu
             } else if (classify(results[k].report, c.device) == PK_DEVICE) {
                 pl.dreport = results[k].report;
             } else if (void *alias = cap <= c.direct_max ? pinned_device_alias(results[k].report) : nullptr) {
-                pl.dreport = static_cast<arc_mismatch_t *>(alias);  // small pinned report: written over PCIe by K2
+                pl.dreport = static_cast<arc_mismatch_t *>(alias);  // small pinned report: written over PCIe by the report phase
             } else {
                 pl.host_report = true;
                 pl.stage_off = stage_entries;
@@ -738,7 +738,7 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
         fprintf(stderr, "[arcv] sms=%d stages=%d ctas/sm=%d (occupancy %d) k2_grid=%d fused=%d regs=%d static_smem=%zu dyn_smem=%zu local=%zu\n",
                 c->num_sms, c->stages, c->ctas_per_sm, occ, c->k2_grid, (int)c->fused, fa.numRegs, fa.sharedSizeBytes, smem, fa.localSizeBytes);
     }
-    // counters: [0] tile tickets, [1] finished CTAs, [2] K2 grid barrier,
+    // counters: [0] tile tickets, [1] finished CTAs, [2] report-phase grid barrier,
     // [3] 2 x u32 active-list lengths, [4] 2 x u32 pool lengths (by parity),
     // [5] peer-exchange finished blocks
     e = cudaMalloc(&c->counters, 8 * sizeof(unsigned long long));

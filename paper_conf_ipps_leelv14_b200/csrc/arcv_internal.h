@@ -35,9 +35,9 @@ struct Ctx {
     unsigned long long ticket_base = 0, done_base = 0;
 
     uint32_t *tile_cnt = nullptr;      size_t tile_cnt_cap = 0;   // per-tile counts (kept zero)
-    uint64_t *active = nullptr;        size_t active_cap = 0;     // K2 active list (2 words / entry)
+    uint64_t *active = nullptr;        size_t active_cap = 0;     // report-phase active list (2 words / entry)
     uint32_t *active_cnt = nullptr;                               // [2] by parity
-    uint64_t *nz_list = nullptr;                                  // K1 -> K2 pool (kPoolCap entries)
+    uint64_t *nz_list = nullptr;                                  // K1 -> report-phase pool (kPoolCap entries)
     uint32_t *nz_cnt = nullptr;                                   // [2] by parity
     unsigned long long gbar_base = 0;
     uint32_t *group_cnt = nullptr;     size_t group_cap = 0;      // [2][group_cap], parity per K1

@@ -10,7 +10,7 @@
 // owns a symmetric "window" in its HBM, mapped into every other rank with CUDA
 // IPC, and one kernel per call does the whole exchange on the device:
 //
-//   K1/K2 (arcv_device.cuh) write the rank's local report straight into its own
+//   K1 (arcv_device.cuh) writes the rank's local report straight into its own
 //   window (packet[parity]) and the local summary into a device mirror;
 //   arcv_peer_kernel then
 //     1. publishes: block 0 writes the local header into its window, fences at
@@ -211,7 +211,7 @@ void peer_finalize(Ctx &c) {
     c.peer_ready = false;
 }
 
-// The sharded compare over the peer windows: local K1/K2 into the own window,
+// The sharded compare over the peer windows: local K1 into the own window,
 // then one exchange+merge kernel, then one wait.
 int peer_compare(Ctx &c, const arc_verify_region_t &r, arc_verify_result_t *result) {
     int st = validate_region(r.out, r.ref, r.n, r.dtype, r.abs_tol, r.rel_tol, r.max_report, result);

@@ -16,15 +16,15 @@ constexpr int kThreads = kConsumerThreads + 32;     // + producer warp
 constexpr int kVecPerThread = kTileBytes / 16 / kConsumerThreads;  // 4
 constexpr int kMaxInlineSegs = 16;                 // regions passed as kernel parameters (C3: 12)
 constexpr int kGroupTiles = 256;                    // tiles per group counter
-constexpr int kPoolCap = 2048;                      // K2 pool path: max listed nonzero tiles
-constexpr uint64_t kDirectDyn = 4096;               // sparse reports: K2 writes a pinned host report directly
-constexpr uint64_t kDirectBit = 1ull << 63;         // K2 tile prefix flag: entries go to report_alias
+constexpr int kPoolCap = 2048;                      // report phase, pool path: max listed nonzero tiles
+constexpr uint64_t kDirectDyn = 4096;               // sparse reports: written directly into pinned host memory
+constexpr uint64_t kDirectBit = 1ull << 63;         // report-phase tile prefix flag: entries go to report_alias
 static_assert(kVecPerThread == 4, "packed-scan layout assumes 4 vectors per thread");
-static_assert(kGroupTiles == kConsumerThreads, "K2 scans one group per block pass");
+static_assert(kGroupTiles == kConsumerThreads, "the report phase scans one group per block pass");
 
 constexpr uint32_t kFlagProbe = 2u;       // Params.flags: stream only, no predicate (read probe)
 constexpr uint32_t kSegBaseFromAcc = 1u;  // chunk of a streamed region: prefix base = acc count - own total
-constexpr uint32_t kSegReportHost = 2u;   // `report` is (mapped) host memory: K2's writes need a system-scope release
+constexpr uint32_t kSegReportHost = 2u;   // `report` is (mapped) host memory (ARCV_WRITER_SYS diagnostic)
 
 // One contiguous piece of one region (a whole region, or one chunk of a region
 // streamed from host memory).
@@ -70,15 +70,15 @@ struct Params {
     uint32_t *group_cnt;      // per-group counts of this launch
     uint32_t *group_zero;     // the other parity buffer, zeroed by K1 for the next launch
     uint64_t n_group_zero;
-    uint64_t *active;         // K2 active-tile list: {seg << 40 | tile, prefix}
+    uint64_t *active;         // report-phase active-tile list: {seg << 40 | tile, prefix}
     uint32_t *active_cnt;     // this launch's list length
     uint32_t *active_cnt_zero;  // the other parity, zeroed by K1 for the next launch
-    uint64_t *nz_list;        // K1 -> K2 pool: {seg << 40 | tile, count} of nonzero tiles
+    uint64_t *nz_list;        // K1 -> report phase pool: {seg << 40 | tile, count} of nonzero tiles
     uint32_t *nz_cnt;         // this launch's pool length (may exceed kPoolCap: overflow)
     uint32_t *nz_cnt_zero;    // the other parity
-    int k2;                   // K2 follows this K1 (some segment wants a report)
+    int k2;                   // some segment wants a report (report phase: fused, or K2 follows)
     int fused;                // K1 runs the report phase itself (cooperative launch; no K2)
-    unsigned long long *gbar; // K2 grid barrier counter (monotonic)
+    unsigned long long *gbar; // report-phase grid barrier counter (monotonic)
     unsigned long long gbar_base;
     Acc *acc;
     Acc *result;
