@@ -282,6 +282,34 @@ def test_batch_sparse_region_next_to_dense(av, orc, buf):
     assert_same(g, ea, f"alone {buf}")
 
 
+@pytest.mark.parametrize("buf", ["pinned_small", "pinned_large", "pageable"])
+def test_report_visibility_stress(av, orc, buf):
+    """The host reads report entries written over PCIe by many CTAs, ordered only by the
+    last CTA's cumulative system fence before the completion word: poison the buffer before
+    every call and check every entry, over many back-to-back calls alternating two inputs."""
+    cases = []
+    for seed in (11, 12):
+        reg = synth.configs.Region("S", "f64", 1 << 22, 3000 + seed, 1e-6, 1e-5, 1 << 20, "f64",
+                                   n_inject=300 + seed, n_nan=2)
+        o, r = reg.slice(device="cuda")
+        e = orc.compare(o.cpu().numpy(), r.cpu().numpy(), "f64", 1e-6, 1e-5, 5000)
+        cases.append((o, r, e))
+    cap = {"pinned_small": 5000, "pinned_large": 1 << 17, "pageable": 5000}[buf]
+    if buf == "pageable":
+        rep = np.zeros(cap, dtype=av.REPORT_DTYPE)
+    else:
+        rep = torch.empty(24 * cap, dtype=torch.uint8, pin_memory=True).numpy().view(av.REPORT_DTYPE)
+    calls = [av.prepare(o, r, 1e-6, 1e-5, 5000, report=rep) for o, r, _ in cases]
+    poison = np.frombuffer(b"\xff" * 24, dtype=av.REPORT_DTYPE)[0]
+    for it in range(200):
+        k = it & 1
+        rep[:] = poison
+        g = calls[k]()
+        e = cases[k][2]
+        assert g.n_mismatch == e.n_mismatch and g.n_reported == e.n_reported, it
+        assert np.array_equal(rep[: g.n_reported], e.report), (buf, it)
+
+
 # ----------------------------------------------------------- host inputs
 @pytest.mark.parametrize("where", ["ref_pinned", "both_pinned", "ref_pageable"])
 def test_host_inputs_streamed(av, orc, where):
