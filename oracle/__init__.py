@@ -165,6 +165,33 @@ def merge_shards(parts, max_report: int) -> OracleResult:
     return OracleResult(n, count, max_abs, max_rel, n_rep, report[:n_rep].copy())
 
 
+def compare_threads(out, ref, dtype: str, abs_tol: float, rel_tol: float, max_report: int,
+                    threads: int | None = None, pool=None) -> OracleResult:
+    """The sequential oracle, unchanged, on ``threads`` contiguous chunks at once
+    (host threads: ctypes releases the GIL during each call), merged by
+    ``merge_shards`` -- the same definition as the cross-GPU merge.  Equal to
+    ``compare`` on the whole arrays (pinned in tests/test_oracle.py).  Used only
+    to time the oracle on all host cores (bench.py cpu_baseline / --impl
+    reference)."""
+    from concurrent.futures import ThreadPoolExecutor
+
+    out = np.ascontiguousarray(out).reshape(-1)
+    ref = np.ascontiguousarray(ref).reshape(-1)
+    threads = max(1, int(threads or len(os.sched_getaffinity(0))))
+    n = out.size
+    cuts = [k * n // threads for k in range(threads + 1)]
+
+    def part(k):
+        return compare(out[cuts[k]:cuts[k + 1]], ref[cuts[k]:cuts[k + 1]], dtype, abs_tol, rel_tol, max_report)
+
+    if pool is not None:
+        parts = list(pool.map(part, range(threads)))
+    else:
+        with ThreadPoolExecutor(threads) as ex:
+            parts = list(ex.map(part, range(threads)))
+    return merge_shards(parts, max_report)
+
+
 def checksum(data) -> tuple[int, int]:
     """The N4 debug-assertion checksum (sum, xor) of a host array's bytes."""
     lib = _load()

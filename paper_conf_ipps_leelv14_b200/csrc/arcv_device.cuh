@@ -1140,13 +1140,21 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
                         atomicAdd(p.tile_cnt + g.slot_begin + lt, tc);
                         atomicAdd(p.group_cnt + g.group_begin + lt / kGroupTiles, tc);
                         // short list of nonzero tiles for the pool path (checked
-                        // before the atomic so a dense call stops touching it)
-                        if (*(volatile uint32_t *)p.nz_cnt < (uint32_t)kPoolCap) {
+                        // before the atomic so a dense call stops touching it).
+                        // A tile left out must leave the count ABOVE kPoolCap:
+                        // a count of exactly kPoolCap means "all listed", so a
+                        // tile that finds the list full lifts it to kPoolCap + 1
+                        // (without this, 2049 nonzero tiles could end with a
+                        // count of 2048 and take the pool path one tile short).
+                        const uint32_t v = *(volatile uint32_t *)p.nz_cnt;
+                        if (v < (uint32_t)kPoolCap) {
                             const uint32_t k = atomicAdd(p.nz_cnt, 1u);
                             if (k < (uint32_t)kPoolCap) {
                                 p.nz_list[2 * k] = ((uint64_t)si.seg << 40) | lt;
                                 p.nz_list[2 * k + 1] = tc;
                             }
+                        } else if (v == (uint32_t)kPoolCap) {
+                            atomicMax(p.nz_cnt, (uint32_t)kPoolCap + 1u);
                         }
                     }
                 }

@@ -262,6 +262,21 @@ def test_shard_merge_equals_unsharded(oracle_mod, p, max_report):
     assert np.array_equal(m.report, full.report)
 
 
+@pytest.mark.parametrize("threads", [1, 3, 8])
+@pytest.mark.parametrize("max_report", [0, 7, 45, 1 << 20])
+def test_threaded_oracle_equals_sequential(oracle_mod, threads, max_report):
+    """compare_threads (the oracle on contiguous chunks in host threads + merge_shards, used
+    only to time the oracle on all cores) returns exactly the sequential oracle's result."""
+    for c, dt in ((synth.C1(), "f32"), (synth.C4(1 << 18), "f64"), (synth.C5(1 << 16), "i32")):
+        out, ref = c.slice()
+        out, ref = out.numpy(), ref.numpy()
+        full = oracle_mod.compare(out, ref, dt, c.abs_tol, c.rel_tol, max_report)
+        m = oracle_mod.compare_threads(out, ref, dt, c.abs_tol, c.rel_tol, max_report, threads=threads)
+        assert (m.n, m.n_mismatch, m.n_reported) == (full.n, full.n_mismatch, full.n_reported)
+        assert m.max_abs_err == full.max_abs_err and m.max_rel_err == full.max_rel_err
+        assert np.array_equal(m.report, full.report)
+
+
 # ---------------------------------------------------------------- generator
 def test_generator_pinned_to_python():
     idx = torch.tensor([0, 1, 2, 3, 99991, (1 << 33) + 5], dtype=torch.int64)
