@@ -310,6 +310,30 @@ def test_report_visibility_stress(av, orc, buf):
         assert np.array_equal(rep[: g.n_reported], e.report), (buf, it)
 
 
+def test_randomized_fuzz(av, orc):
+    """Seeded fuzz: dtype, length, mismatch density (around the 2048-tile pool boundary and
+    dense), element offset, max_report and report-buffer kind drawn at random; every call
+    bit-exact against the oracle."""
+    rng = np.random.default_rng(20141)
+    pinned = torch.empty(24 * 70000, dtype=torch.uint8, pin_memory=True).numpy().view(av.REPORT_DTYPE)
+    dev_rep = torch.empty(24 * 70000, dtype=torch.uint8, device="cuda")
+    for it in range(60):
+        dt = ["f32", "f64", "i32", "i64", "u8"][int(rng.integers(5))]
+        te = TILE_ELEMS[dt]
+        n = int(rng.integers(1, 3000)) * te // 2 + int(rng.integers(0, te))
+        off = int(rng.integers(0, 3))
+        rate = float(rng.choice([0.0, 1e-5, 3e-4, 1e-3, 0.05, 0.5]))
+        o, r = random_pair(dt, n + off, seed=5000 + it, rate=rate)
+        o, r = o[off:], r[off:]
+        mr = int(rng.choice([0, 1, 100, 4096, 60000]))
+        kind = int(rng.integers(3))
+        rep = (None, pinned, dev_rep)[kind]
+        e = orc.compare(o.cpu().numpy(), r.cpu().numpy(), dt, 1e-6, 1e-5, mr)
+        for rep_call in range(2):
+            g = av.compare(o, r, 1e-6, 1e-5, mr, report=rep)
+            assert_same(g, e, f"it={it} dt={dt} n={n} off={off} rate={rate} mr={mr} kind={kind} call={rep_call}")
+
+
 # ----------------------------------------------------------- host inputs
 @pytest.mark.parametrize("where", ["ref_pinned", "both_pinned", "ref_pageable"])
 def test_host_inputs_streamed(av, orc, where):
