@@ -334,6 +334,33 @@ def test_randomized_fuzz(av, orc):
             assert_same(g, e, f"it={it} dt={dt} n={n} off={off} rate={rate} mr={mr} kind={kind} call={rep_call}")
 
 
+def test_randomized_fuzz_batch_and_host(av, orc):
+    """Seeded fuzz over batches (1-20 random regions, mixed dtypes and densities, one grid)
+    and host-resident inputs (pinned out/ref streamed in chunks: per-chunk report bases)."""
+    rng = np.random.default_rng(20142)
+    for it in range(25):
+        regs, exps = [], []
+        for k in range(int(rng.integers(1, 21))):
+            dt = ["f32", "f64", "i32", "i64", "u8"][int(rng.integers(5))]
+            n = int(rng.integers(0, 200_000))
+            rate = float(rng.choice([0.0, 1e-4, 0.01, 0.3]))
+            o, r = random_pair(dt, n, seed=7000 + 50 * it + k, rate=rate)
+            mr = int(rng.choice([0, 3, 500, 100000]))
+            regs.append((o, r, 1e-6, 1e-5, mr))
+            exps.append(orc.compare(o.cpu().numpy(), r.cpu().numpy(), dt, 1e-6, 1e-5, mr))
+        for g, e in zip(av.batch(regs), exps):
+            assert_same(g, e, f"batch it={it}")
+    for it in range(8):
+        dt = ["f32", "f64", "i32"][it % 3]
+        n = int(rng.integers(1, 40)) * (1 << 20) // 3 + int(rng.integers(0, 5000))
+        o, r = random_pair(dt, n, seed=9000 + it, rate=float(rng.choice([1e-6, 1e-4, 0.02])))
+        mr = int(rng.choice([10, 5000, 1 << 20]))
+        e = orc.compare(o.cpu().numpy(), r.cpu().numpy(), dt, 1e-6, 1e-5, mr)
+        ho, hr = o.cpu().pin_memory(), r.cpu().pin_memory()
+        for a, b, where in ((o, hr, "ref on host"), (ho, hr, "both on host")):
+            assert_same(av.compare(a, b, 1e-6, 1e-5, mr), e, f"host it={it} {where} n={n} mr={mr}")
+
+
 # ----------------------------------------------------------- host inputs
 @pytest.mark.parametrize("where", ["ref_pinned", "both_pinned", "ref_pageable"])
 def test_host_inputs_streamed(av, orc, where):
