@@ -73,3 +73,34 @@ def test_kernel_flags_in_build_log(lib):
     for flag in ("-fmad=false", "-ftz=false", "-prec-div=true", "arch=compute_100a,code=sm_100a"):
         assert flag in first
     assert "use_fast_math" not in first
+
+
+def _build_c_example(out_path):
+    import subprocess
+
+    cmd = ["gcc", "-std=c99", "-O2", "-Wall", "-Werror", "-I", os.path.join(ROOT, "include"),
+           "-I", "/usr/local/cuda/include", os.path.join(ROOT, "examples", "verify_region.c"),
+           "-L", os.path.join(ROOT, "paper_conf_ipps_leelv14_b200"), "-larcverify",
+           "-L", "/usr/local/cuda/lib64", "-lcudart",
+           "-Wl,-rpath," + os.path.join(ROOT, "paper_conf_ipps_leelv14_b200"), "-lm", "-o", out_path]
+    return subprocess.run(cmd, capture_output=True, text=True)
+
+
+def test_c_example_compiles_and_links_as_c99(lib, tmp_path):
+    """The ABI is plain C: a C99 program includes the header and links the library."""
+    r = _build_c_example(str(tmp_path / "verify_region"))
+    assert r.returncode == 0, r.stderr
+
+
+@pytest.mark.gpu
+def test_c_example_runs(lib, tmp_path):
+    """The C program verifies a region on the GPU and finds exactly the planted stale row."""
+    import subprocess
+
+    exe = str(tmp_path / "verify_region")
+    r = _build_c_example(exe)
+    assert r.returncode == 0, r.stderr
+    p = subprocess.run([exe], capture_output=True, text=True, timeout=120)
+    assert p.returncode == 0, p.stdout + p.stderr
+    assert "PASS: 998 mismatches" in p.stdout
+    assert "main_kernel0" in p.stdout
