@@ -40,6 +40,7 @@
 #include <math_constants.h>
 
 #include "arc_verify.h"
+#include "arcv_exchange.cuh"
 #include "arcv_types.h"
 
 namespace arcv {
@@ -605,6 +606,20 @@ __device__ __forceinline__ void finalize_launch(const Params &p, int tid, int nt
     if (last_cta(p, tid, nthreads, s_last, wrote_host, base) && do_publish) publish(p, tid, nthreads);
 }
 
+// Sharded call with the exchange fused into K1 (p.xfused; K1 is a cooperative
+// launch): the CTA that published the local result (`leader`) publishes the
+// rank's header and flags, then every CTA runs the exchange body -- wait for
+// the peers' flags, merge its share of the global report, and the last one
+// writes the global result and the completion word.  Scratch: the (free)
+// stage memory.
+__device__ __forceinline__ void exchange_tail(const Params &p, int tid, bool leader, uint8_t *smem) {
+    if (leader && tid == 0) {
+        const Acc a = p.mirror[0];  // this thread wrote it in publish()
+        peer_publish_header(p.x, a.count, a.max_abs_bits, a.max_rel_bits);
+    }
+    peer_exchange_body(p.x, tid, *reinterpret_cast<ExShared *>(smem));
+}
+
 // ------------------------------------------------------ report-phase helpers
 // Exclusive scan over the 256 consumer threads (named barrier 1; `tid` = the
 // consumer index, so K1's consumer warps can run it too) of a u64; returns the
@@ -1017,6 +1032,7 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
         const bool last = last_cta(p, tid, kConsumerThreads, &sh.last, wrote_host, done_base);
         if (tid == 0) ARCV_STAMP(1, 11);
         if (last && !(k1_published_if_empty && n_nz == 0)) publish(p, tid, kConsumerThreads);
+        if (p.xfused) exchange_tail(p, tid, last, smem);
     }
     if (tid == 0) ARCV_STAMP(1, 7);
 }
@@ -1194,6 +1210,7 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
         fence_gpu();
         if (p.finalize && (!p.k2 || *(volatile uint32_t *)p.nz_cnt == 0u)) publish(p, ctid, kConsumerThreads);
     }
+    if (p.xfused) exchange_tail(p, ctid, s_last != 0, smem);  // count-only sharded call (no K2 then)
     if (ctid == 0) ARCV_STAMP(0, 3);
 }
 

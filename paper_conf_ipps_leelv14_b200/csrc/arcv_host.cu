@@ -283,7 +283,9 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
     p.flags = (uint32_t)c.flags;
     // ARCV_FLAGS bit 3 (diagnostic): stream sync; deferred (peer) calls wake on the exchange kernel
     p.done_flag = ((c.flags & 8) || c.defer_wait) ? nullptr : c.flag_dev;
-    if (finalize) p.seq = ++c.seq;  // the host waits for the last finalize launch's number
+    // the host waits for the last finalize launch's number (deferred calls wake
+    // on the exchange, which carries its own number)
+    if (finalize && !c.defer_wait) p.seq = ++c.seq;
     p.mirror = finalize ? c.mirror_next : nullptr;
 
     const uint64_t max_grid = (uint64_t)c.num_sms * (uint64_t)c.ctas_per_sm;
@@ -293,9 +295,17 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
     // fused: K1 runs the report phase after a grid barrier (cooperative launch)
     const bool fused = need_compact && c.fused;
     p.fused = fused ? 1 : 0;
+    // fused exchange (sharded peer call): the shard's final launch runs the
+    // exchange in its tail -- cooperative too (its CTAs wait for the peers)
+    const bool xf = c.x_next != nullptr && finalize && (!need_compact || fused);
+    p.xfused = xf ? 1 : 0;
+    if (xf) {
+        p.x = *c.x_next;
+        p.x.done_base = c.peer_done_base;
+    }
     if (timed) CK(cudaEventRecord(c.ev[c.n_ev][0], c.stream));
     cudaError_t e;
-    if (fused) {
+    if (fused || xf) {
         cudaLaunchConfig_t cfg = {};
         cfg.gridDim = dim3(grid);
         cfg.blockDim = dim3(kThreads);
@@ -315,6 +325,10 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
     }
     c.launches++;
     c.ticket_base += tiles + grid;
+    if (xf) {
+        c.peer_done_base += grid;  // every K1 CTA counts once on the exchange counter
+        c.x_taken = true;
+    }
     if (fused) {
         // grid barrier + (finalize) the report phase's completion count
         c.done_base += (uint64_t)grid * (finalize ? 2u : 1u);
@@ -732,6 +746,8 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
     // the report phase runs in K1's tail when its stage memory holds the
     // report phase's (>= 3 stages); ARCV_FUSED=0 forces the separate K2
     c->fused = env_int("ARCV_FUSED", 1) != 0 && smem >= (size_t)kReportSmem;
+    // the exchange in K1's tail needs its scratch in the stage memory
+    c->fused_exchange = env_int("ARCV_FUSED_EXCHANGE", 1) != 0 && smem >= sizeof(ExShared);
     if (env_int("ARCV_VERBOSE", 0)) {
         cudaFuncAttributes fa;
         CK(cudaFuncGetAttributes(&fa, kf));

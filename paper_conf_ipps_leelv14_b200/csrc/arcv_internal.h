@@ -76,6 +76,9 @@ struct Ctx {
 
     // peer-memory exchange (arcv_peer.cu): symmetric windows over NVLink P2P
     bool defer_wait = false;           // run_local: enqueue only (the exchange kernel follows)
+    const PeerParams *x_next = nullptr;  // launch_segments: run this exchange in K1's tail (fused)
+    bool x_taken = false;              // ... and it did (else the exchange kernel runs)
+    bool fused_exchange = true;        // ARCV_FUSED_EXCHANGE=0: always the separate exchange kernel
     Acc *mirror_next = nullptr;        // launch_segments: device copy of the finalised slots
     Acc *mirror = nullptr;             // [1] device
     uint8_t *win = nullptr;            // own window (cudaMalloc, IPC-exported)

@@ -40,151 +40,21 @@
 #include <cstring>
 
 #include "arc_verify.h"
+#include "arcv_exchange.cuh"
 #include "arcv_internal.h"
 
 namespace arcv {
 
-constexpr size_t kFlagBytes = 2 * kMaxRanks * sizeof(unsigned long long);  // [2 parities][kMaxRanks]
-constexpr unsigned long long kPeerTimeoutNs = 60ull * 1000 * 1000 * 1000;  // 60 s
-
-__host__ __device__ inline size_t packet_stride(uint64_t cap) {
-    return (sizeof(arc_shard_header_t) + (size_t)cap * sizeof(arc_mismatch_t) + 127) & ~(size_t)127;
-}
-__host__ __device__ inline unsigned long long *flag_slot(uint8_t *win, int par, int r) {
-    return reinterpret_cast<unsigned long long *>(win) + (size_t)par * kMaxRanks + r;
-}
-__host__ __device__ inline uint8_t *packet_at(uint8_t *win, uint64_t cap, int par) {
-    return win + kFlagBytes + (size_t)par * packet_stride(cap);
-}
-
-struct PeerParams {
-    uint8_t *const *win;            // [p] window base pointers (own + IPC-mapped peers)
-    int rank, p, par;
-    unsigned long long s;           // collective sequence number = flag value
-    uint64_t n_local, max_report, cap;
-    const Acc *mirror;              // local summary (written by the local compare)
-    arc_mismatch_t *dst;            // global report target (device memory or HBM staging), or nullptr
-    arc_mismatch_t *dst_alias;      // device alias of the caller's pinned host report, or nullptr:
-                                    // used instead of dst when the global report has <= kDirectDyn
-                                    // entries (the host then skips its D2H copy; same rule there)
-    arc_shard_header_t *out;        // mapped host: [0] global header, [1].n = status (1 = timeout)
-    unsigned long long *done;       // monotonic finished-block counter
-    unsigned long long done_base;
-    unsigned long long *done_flag;  // mapped completion word
-    unsigned long long seq;
-};
-
-__device__ __forceinline__ void st_release_sys(unsigned long long *p, unsigned long long v) {
-    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long *p) {
-    unsigned long long v;
-    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-    return v;
-}
-// message-passing fences (no fence.sc needed; see arcv_device.cuh fence_gpu/fence_sys)
-__device__ __forceinline__ void peer_fence_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
-__device__ __forceinline__ void peer_fence_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
-__device__ __forceinline__ unsigned long long ld_volatile(const unsigned long long *p) {
-    return *reinterpret_cast<const volatile unsigned long long *>(p);
-}
-__device__ __forceinline__ unsigned long long globaltimer() {
-    unsigned long long t;
-    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-    return t;
-}
-
+// The stand-alone exchange kernel: a programmatic dependent of the local
+// compare (K1), used when K1 did not run the exchange itself (empty or
+// host-streamed shard, ARCV_FUSED_EXCHANGE=0).  Block 0 publishes the header
+// from the local summary mirror; every block then runs the common body.
 __global__ void __launch_bounds__(256) arcv_peer_kernel(const __grid_constant__ PeerParams q) {
-    __shared__ arc_shard_header_t hdr[kMaxRanks];
-    __shared__ arc_shard_plan_t plan[kMaxRanks];
-    __shared__ uint64_t cum[kMaxRanks + 1];
-    __shared__ arc_shard_header_t glob;
-    __shared__ int s_ok, s_last;
-    const int tid = threadIdx.x;
-    uint8_t *own = q.win[q.rank];
+    __shared__ ExShared sh;
     asm volatile("griddepcontrol.wait;" ::: "memory");  // the local compare has completed
-
-    // 1. publish (one thread of the grid)
-    if (blockIdx.x == 0 && tid == 0) {
-        unsigned long long *h = reinterpret_cast<unsigned long long *>(packet_at(own, q.cap, q.par));
-        h[0] = q.n_local;
-        h[1] = q.mirror->count;
-        h[2] = q.mirror->max_abs_bits;
-        h[3] = q.mirror->max_rel_bits;
-        peer_fence_sys();  // header + the local report (previous kernels) before the flags
-        for (int r = 0; r < q.p; ++r) st_release_sys(flag_slot(q.win[r], q.par, q.rank), q.s);
-    }
-    // 2. wait for every rank's flag in the own window
-    if (tid == 0) {
-        int ok = 1;
-        const unsigned long long t0 = globaltimer();
-        for (int r = 0; r < q.p && ok; ++r) {
-            const unsigned long long *f = flag_slot(own, q.par, r);
-            while (ld_acquire_sys(f) != q.s) {
-                if (globaltimer() - t0 > kPeerTimeoutNs) {
-                    ok = 0;
-                    break;
-                }
-                __nanosleep(128);
-            }
-        }
-        s_ok = ok;
-    }
-    __syncthreads();
-    const bool ok = s_ok != 0;
-    uint64_t total = 0;
-    if (ok) {
-        // 3. merge: headers from every window (P2P loads, not cached in L1)
-        for (int r = tid; r < q.p; r += blockDim.x) {
-            const unsigned long long *h = reinterpret_cast<const unsigned long long *>(packet_at(q.win[r], q.cap, q.par));
-            hdr[r].n = ld_volatile(h);
-            hdr[r].n_mismatch = ld_volatile(h + 1);
-            hdr[r].max_abs_bits = ld_volatile(h + 2);
-            hdr[r].max_rel_bits = ld_volatile(h + 3);
-        }
-        __syncthreads();
-        if (tid == 0) {
-            merge_plan_impl(hdr, q.p, q.max_report, plan, &glob);
-            cum[0] = 0;
-            for (int r = 0; r < q.p; ++r) cum[r + 1] = cum[r] + plan[r].contrib;
-        }
-        __syncthreads();
-        total = q.dst ? cum[q.p] : 0;
-        arc_mismatch_t *const dst = (q.dst_alias && total <= kDirectDyn) ? q.dst_alias : q.dst;
-        for (uint64_t gi = (uint64_t)blockIdx.x * blockDim.x + tid; gi < total;
-             gi += (uint64_t)gridDim.x * blockDim.x) {
-            int lo = 0, hi = q.p;  // last r with cum[r] <= gi
-            while (hi - lo > 1) {
-                const int mid = (lo + hi) >> 1;
-                if (cum[mid] <= gi) lo = mid; else hi = mid;
-            }
-            const uint64_t j = gi - cum[lo];
-            const unsigned long long *src = reinterpret_cast<const unsigned long long *>(
-                packet_at(q.win[lo], q.cap, q.par) + sizeof(arc_shard_header_t) + j * sizeof(arc_mismatch_t));
-            arc_mismatch_t e;
-            e.index = ld_volatile(src) + plan[lo].index_offset;
-            e.out_bits = ld_volatile(src + 1);
-            e.ref_bits = ld_volatile(src + 2);
-            dst[plan[lo].prefix + j] = e;
-        }
-    }
-    // 4. completion: the last block publishes the global header, then the word
-    __syncthreads();
-    if (tid == 0) {
-        if (!ok) q.out[1].n = 1;  // status: timed out
-        // gpu-scope release: the last block's system fence below is cumulative
-        // (entries written to a pinned host report included)
-        peer_fence_gpu();
-        const unsigned long long prev = atomicAdd(q.done, 1ull);
-        s_last = (prev - q.done_base) == (unsigned long long)(gridDim.x - 1);
-    }
-    __syncthreads();
-    if (s_last && tid == 0) {
-        peer_fence_gpu();
-        if (ok) q.out[0] = glob;
-        peer_fence_sys();
-        *(volatile unsigned long long *)q.done_flag = q.seq;
-    }
+    if (blockIdx.x == 0 && threadIdx.x == 0)
+        peer_publish_header(q, q.mirror->count, q.mirror->max_abs_bits, q.mirror->max_rel_bits);
+    peer_exchange_body(q, (int)threadIdx.x, sh);
 }
 
 // ------------------------------------------------------------------- host
@@ -211,8 +81,10 @@ void peer_finalize(Ctx &c) {
     c.peer_ready = false;
 }
 
-// The sharded compare over the peer windows: local K1 into the own window,
-// then one exchange+merge kernel, then one wait.
+// The sharded compare over the peer windows: local K1 into the own window and
+// -- fused, the default -- the exchange in the same kernel's tail (K1 is then a
+// cooperative launch: its CTAs wait for the peers' flags), else one
+// exchange+merge kernel after it; then one wait.
 int peer_compare(Ctx &c, const arc_verify_region_t &r, arc_verify_result_t *result) {
     int st = validate_region(r.out, r.ref, r.n, r.dtype, r.abs_tol, r.rel_tol, r.max_report, result);
     if (st) return st;
@@ -221,16 +93,6 @@ int peer_compare(Ctx &c, const arc_verify_region_t &r, arc_verify_result_t *resu
     arc_mismatch_t *entries =
         reinterpret_cast<arc_mismatch_t *>(packet_at(c.win, c.win_cap, par) + sizeof(arc_shard_header_t));
     if (r.n == 0) CK(cudaMemsetAsync(c.mirror, 0, sizeof(Acc), c.stream));
-    // local a1-a6 on the shard, enqueue only; the report goes to the own window
-    arc_verify_result_t local;
-    memset(&local, 0, sizeof(local));
-    local.report = entries;
-    c.defer_wait = true;
-    c.mirror_next = c.mirror;
-    st = run_local(c, &r, 1, &local, &entries, false, nullptr);
-    c.defer_wait = false;
-    c.mirror_next = nullptr;
-    if (st) return st;
     // global report target
     arc_mismatch_t *dst = nullptr;
     bool host_report = false;
@@ -257,21 +119,40 @@ int peer_compare(Ctx &c, const arc_verify_region_t &r, arc_verify_result_t *resu
     q.done_base = c.peer_done_base;
     q.done_flag = c.flag_dev;
     q.seq = ++c.seq;
-    // a few blocks: the merge moves <= max_report x 24 B, mostly a handful
-    const uint64_t work = std::min<uint64_t>(r.max_report, 1ull << 40);
-    const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(32, (work + 2047) / 2048));
-    cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3(grid);
-    cfg.blockDim = dim3(256);
-    cfg.stream = c.stream;
-    cudaLaunchAttribute at[1];
-    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    at[0].val.programmaticStreamSerializationAllowed = 1;
-    cfg.attrs = at;
-    cfg.numAttrs = c.pdl ? 1 : 0;
-    CK(cudaLaunchKernelEx(&cfg, arcv_peer_kernel, q));
-    c.launches++;
-    c.peer_done_base += (unsigned long long)grid;
+    // the fused exchange needs a local launch: a non-empty, device-resident shard
+    const bool want_fused = c.fused_exchange && r.n > 0 && classify(r.out, c.device) == PK_DEVICE &&
+                            classify(r.ref, c.device) == PK_DEVICE;
+    // local a1-a6 on the shard, enqueue only; the report goes to the own window
+    arc_verify_result_t local;
+    memset(&local, 0, sizeof(local));
+    local.report = entries;
+    c.defer_wait = true;
+    c.mirror_next = c.mirror;
+    c.x_next = want_fused ? &q : nullptr;
+    c.x_taken = false;
+    st = run_local(c, &r, 1, &local, &entries, false, nullptr);
+    c.defer_wait = false;
+    c.mirror_next = nullptr;
+    c.x_next = nullptr;
+    if (st) return st;
+    if (!c.x_taken) {
+        // a few blocks: the merge moves <= max_report x 24 B, mostly a handful
+        q.done_base = c.peer_done_base;
+        const uint64_t work = std::min<uint64_t>(r.max_report, 1ull << 40);
+        const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(32, (work + 2047) / 2048));
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(grid);
+        cfg.blockDim = dim3(256);
+        cfg.stream = c.stream;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        at[0].val.programmaticStreamSerializationAllowed = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = c.pdl ? 1 : 0;
+        CK(cudaLaunchKernelEx(&cfg, arcv_peer_kernel, q));
+        c.launches++;
+        c.peer_done_base += (unsigned long long)grid;
+    }
     st = wait_results(c);
     if (st) return st;
     if (c.peer_out_host[1].n != 0) {

@@ -57,6 +57,25 @@ struct Acc {  // per-region accumulators / result slot, 32 bytes
     unsigned long long pad;
 };
 
+// The sharded exchange over peer windows (arcv_exchange.cuh): one call's
+// parameters, used by the exchange kernel and by K1's fused exchange.
+struct PeerParams {
+    uint8_t *const *win;            // [p] window base pointers (own + IPC-mapped peers)
+    int rank, p, par;
+    unsigned long long s;           // collective sequence number = flag value
+    uint64_t n_local, max_report, cap;
+    const Acc *mirror;              // local summary (written by the local compare)
+    arc_mismatch_t *dst;            // global report target (device memory or HBM staging), or nullptr
+    arc_mismatch_t *dst_alias;      // device alias of the caller's pinned host report, or nullptr:
+                                    // used instead of dst when the global report has <= kDirectDyn
+                                    // entries (the host then skips its D2H copy; same rule there)
+    arc_shard_header_t *out;        // mapped host: [0] global header, [1].n = status (1 = timeout)
+    unsigned long long *done;       // monotonic finished-block counter
+    unsigned long long done_base;
+    unsigned long long *done_flag;  // mapped completion word
+    unsigned long long seq;
+};
+
 struct Params {
     const Seg *segs;          // device table, or nullptr -> inline_segs
     uint32_t n_segs;
@@ -88,6 +107,8 @@ struct Params {
     uint32_t report_host;           // some report lives in pinned host memory (system-scope fences)
     int finalize;
     uint32_t flags;
+    int xfused;                     // sharded call: K1's CTAs run the exchange after the local result
+    PeerParams x;                   // its parameters (xfused only)
     Seg inline_segs[kMaxInlineSegs];
 };
 

@@ -104,11 +104,14 @@ def _worker(rank, world, port, q):
 
 
 @pytest.mark.timeout(600)
-@pytest.mark.parametrize("world", [2, 3])
-def test_peer_exchange_matches_unsharded_oracle(world):
+@pytest.mark.parametrize("world,fused", [(2, "1"), (3, "1"), (2, "0")])
+def test_peer_exchange_matches_unsharded_oracle(world, fused, monkeypatch):
+    """fused = 1: the exchange runs in K1's tail (one kernel per call); 0: the separate
+    exchange kernel (also what empty shards use)."""
     import oracle
 
     oracle.build()
+    monkeypatch.setenv("ARCV_FUSED_EXCHANGE", fused)  # inherited by the spawned ranks
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
