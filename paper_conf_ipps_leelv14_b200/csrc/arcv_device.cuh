@@ -1041,9 +1041,11 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
 // grid barrier), a programmatic dependent of K1.  Used when the fused tail does
 // not fit K1's stage memory (fewer than 3 stages) or ARCV_FUSED=0.
 // grid: SMs x co-resident CTAs; block: 256; dynamic smem: kReportSmem.
-__global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __grid_constant__ Params p) {
+template <int NSEG>
+__global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __grid_constant__ ParamsN<NSEG> pn) {
     extern __shared__ __align__(128) uint8_t smem[];
-    const Seg *segs = p.segs ? p.segs : p.inline_segs;
+    const Params &p = pn;
+    const Seg *segs = p.segs ? p.segs : pn.inline_segs;
     if (threadIdx.x == 0) ARCV_STAMP(1, 0);
     // wait for K1's completion (and the visibility of its writes) before
     // touching any of them
@@ -1054,8 +1056,9 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
 
 
 // ------------------------------------------------------------------ K1: stream
-template <int S, int MINB>
-__global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __grid_constant__ Params p) {
+template <int S, int MINB, int NSEG>
+__global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __grid_constant__ ParamsN<NSEG> pn) {
+    const Params &p = pn;
     extern __shared__ __align__(128) uint8_t smem[];
     __shared__ __align__(8) uint64_t full_bar[S];
     __shared__ __align__(8) uint64_t empty_bar[S];
@@ -1065,7 +1068,7 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
     __shared__ int s_last;
     __shared__ uint32_t s_tile[S];
 
-    const Seg *segs = p.segs ? p.segs : p.inline_segs;
+    const Seg *segs = p.segs ? p.segs : pn.inline_segs;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
     if (threadIdx.x == 0) {

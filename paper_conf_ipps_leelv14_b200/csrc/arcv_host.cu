@@ -44,16 +44,70 @@ int cuda_fail(cudaError_t e, const char *what) {
 Ctx *g_ctx = nullptr;
 
 // ------------------------------------------------------------------ kernels
-typedef void (*KernelFn)(Params);
+template <int NSEG>
+using KernelFnN = void (*)(ParamsN<NSEG>);
 // Variants: (stages, min CTAs per SM).  Stage ring bytes per SM stay within
-// the 228 KB shared memory: 3x2 (default), 2x3, 4x1, 6x1.
-static KernelFn stream_kernel_for(int s) {
+// the 228 KB shared memory: 3x2 (default), 2x3, 4x1, 6x1.  NSEG: inline
+// segments in the parameter block (1 or kMaxInlineSegs).
+template <int NSEG>
+static KernelFnN<NSEG> stream_kernel_for(int s) {
     switch (s) {
-        case 2: return arcv_stream_kernel<2, 3>;
-        case 4: return arcv_stream_kernel<4, 1>;
-        case 6: return arcv_stream_kernel<6, 1>;
-        default: return arcv_stream_kernel<3, 2>;
+        case 2: return arcv_stream_kernel<2, 3, NSEG>;
+        case 4: return arcv_stream_kernel<4, 1, NSEG>;
+        case 6: return arcv_stream_kernel<6, 1, NSEG>;
+        default: return arcv_stream_kernel<3, 2, NSEG>;
     }
+}
+
+// Launch K1 (cooperative when `coop`) and, when `k2`, the separate report
+// kernel, with a parameter block of NSEG inline segments.
+template <int NSEG>
+static cudaError_t launch_k1_k2(const Params &base, const Seg *inl, uint32_t n_inl, uint32_t grid, size_t smem,
+                                cudaStream_t st, bool coop, bool k2, uint32_t grid2, bool *pdl, const Params *k2p) {
+    ParamsN<NSEG> pn;
+    static_cast<Params &>(pn) = base;
+    if (n_inl) memcpy(pn.inline_segs, inl, n_inl * sizeof(Seg));
+    cudaError_t e;
+    if (coop) {
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(grid);
+        cfg.blockDim = dim3(kThreads);
+        cfg.dynamicSmemBytes = smem;
+        cfg.stream = st;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeCooperative;
+        at[0].val.cooperative = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        e = cudaLaunchKernelEx(&cfg, stream_kernel_for<NSEG>(g_ctx->stages), pn);
+    } else {
+        stream_kernel_for<NSEG>(g_ctx->stages)<<<grid, kThreads, smem, st>>>(pn);
+        e = cudaGetLastError();
+    }
+    if (e != cudaSuccess || !k2) return e;
+    static_cast<Params &>(pn) = *k2p;
+    // cooperative (the group path has a grid barrier) and, unless disabled, a
+    // programmatic dependent of K1: its launch overlaps K1's tail
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid2);
+    cfg.blockDim = dim3(kConsumerThreads);
+    cfg.dynamicSmemBytes = kReportSmem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[2];
+    at[0].id = cudaLaunchAttributeCooperative;
+    at[0].val.cooperative = 1;
+    at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[1].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = *pdl ? 2 : 1;
+    e = cudaLaunchKernelEx(&cfg, arcv_compact_kernel<NSEG>, pn);
+    if (e != cudaSuccess && *pdl) {  // PDL refused with a cooperative launch: plain cooperative
+        cudaGetLastError();
+        *pdl = false;
+        cfg.numAttrs = 1;
+        e = cudaLaunchKernelEx(&cfg, arcv_compact_kernel<NSEG>, pn);
+    }
+    return e;
 }
 
 static int env_int(const char *name, int dflt) {
@@ -240,8 +294,7 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
             segs[k].flags |= kSegReportHost;
         }
     if (n_segs <= (uint32_t)kMaxInlineSegs) {
-        memcpy(p.inline_segs, segs, n_segs * sizeof(Seg));
-        p.segs = nullptr;
+        p.segs = nullptr;  // inline (copied into the parameter block at launch)
     } else {
         st = grow_device(&c.seg_dev, &c.seg_dev_cap, n_segs, false, c.stream);
         if (st) return st;
@@ -303,27 +356,23 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
         p.x = *c.x_next;
         p.x.done_base = c.peer_done_base;
     }
-    if (timed) CK(cudaEventRecord(c.ev[c.n_ev][0], c.stream));
-    cudaError_t e;
-    if (fused || xf) {
-        cudaLaunchConfig_t cfg = {};
-        cfg.gridDim = dim3(grid);
-        cfg.blockDim = dim3(kThreads);
-        cfg.dynamicSmemBytes = smem;
-        cfg.stream = c.stream;
-        cudaLaunchAttribute at[1];
-        at[0].id = cudaLaunchAttributeCooperative;
-        at[0].val.cooperative = 1;
-        cfg.attrs = at;
-        cfg.numAttrs = 1;
-        e = cudaLaunchKernelEx(&cfg, stream_kernel_for(c.stages), p);
-        if (e != cudaSuccess) return cuda_fail(e, "arcv_stream_kernel cooperative launch");
-    } else {
-        stream_kernel_for(c.stages)<<<grid, kThreads, smem, c.stream>>>(p);
-        e = cudaGetLastError();
-        if (e != cudaSuccess) return cuda_fail(e, "arcv_stream_kernel launch");
+    // the separate report kernel (K2) gets the same block with its own bases
+    const bool k2 = need_compact && !fused;
+    const uint32_t grid2 = (uint32_t)c.k2_grid;
+    Params p2;
+    if (k2) {
+        p2 = p;
+        p2.finalize = finalize ? 1 : 0;
+        const unsigned long long k1_done = (p.finalize || p.k2) ? grid : 0;
+        p2.done_base = c.done_base + k1_done;
     }
-    c.launches++;
+    if (timed) CK(cudaEventRecord(c.ev[c.n_ev][0], c.stream));
+    const uint32_t n_inl = p.segs ? 0u : n_segs;
+    cudaError_t e = n_inl > 1
+        ? launch_k1_k2<kMaxInlineSegs>(p, segs, n_inl, grid, smem, c.stream, fused || xf, k2, grid2, &c.pdl, &p2)
+        : launch_k1_k2<1>(p, segs, n_inl, grid, smem, c.stream, fused || xf, k2, grid2, &c.pdl, &p2);
+    if (e != cudaSuccess) return cuda_fail(e, "arcv_stream_kernel / arcv_compact_kernel launch");
+    c.launches += k2 ? 2 : 1;
     c.ticket_base += tiles + grid;
     if (xf) {
         c.peer_done_base += grid;  // every K1 CTA counts once on the exchange counter
@@ -336,33 +385,7 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
     } else if (p.finalize || p.k2) {
         c.done_base += grid;  // K1 counts its CTAs to find its last one
     }
-    if (need_compact && !fused) {
-        p.finalize = finalize ? 1 : 0;
-        p.done_base = c.done_base;
-        const uint32_t grid2 = (uint32_t)c.k2_grid;
-        // cooperative (the group path has a grid barrier) and, unless disabled,
-        // a programmatic dependent of K1: its launch overlaps K1's tail
-        cudaLaunchConfig_t cfg = {};
-        cfg.gridDim = dim3(grid2);
-        cfg.blockDim = dim3(kConsumerThreads);
-        cfg.dynamicSmemBytes = kCompactSmem;
-        cfg.stream = c.stream;
-        cudaLaunchAttribute at[2];
-        at[0].id = cudaLaunchAttributeCooperative;
-        at[0].val.cooperative = 1;
-        at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-        at[1].val.programmaticStreamSerializationAllowed = 1;
-        cfg.attrs = at;
-        cfg.numAttrs = c.pdl ? 2 : 1;
-        e = cudaLaunchKernelEx(&cfg, arcv_compact_kernel, p);
-        if (e != cudaSuccess && c.pdl) {  // PDL refused with a cooperative launch: plain cooperative
-            cudaGetLastError();
-            c.pdl = false;
-            cfg.numAttrs = 1;
-            e = cudaLaunchKernelEx(&cfg, arcv_compact_kernel, p);
-        }
-        if (e != cudaSuccess) return cuda_fail(e, "arcv_compact_kernel cooperative launch");
-        c.launches++;
+    if (k2) {
         c.gbar_base += grid2;
         if (finalize) c.done_base += grid2;
     }
@@ -729,16 +752,20 @@ int arc_verify_init(const arc_verify_opts_t *opts) {
     c->stages = env_int("ARCV_STAGES", 3);
     if (c->stages != 2 && c->stages != 3 && c->stages != 4 && c->stages != 6) c->stages = 3;
     const size_t smem = (size_t)c->stages * kStageBytes;
-    KernelFn kf = stream_kernel_for(c->stages);
+    KernelFnN<kMaxInlineSegs> kf = stream_kernel_for<kMaxInlineSegs>(c->stages);
     CK(cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    CK(cudaFuncSetAttribute(arcv_compact_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kCompactSmem));
+    CK(cudaFuncSetAttribute(stream_kernel_for<1>(c->stages), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    CK(cudaFuncSetAttribute(arcv_compact_kernel<kMaxInlineSegs>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            kCompactSmem));
+    CK(cudaFuncSetAttribute(arcv_compact_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, kCompactSmem));
     int occ = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kf, kThreads, smem));
     if (occ < 1) { set_error("kernel does not fit on an SM (smem %zu)", smem); return ARC_E_UNSUPPORTED; }
     // K2: as many co-resident CTAs as fit (cooperative launch), so the re-read
     // tiles of a sparse report are all in flight in one wave
     int occ2 = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, arcv_compact_kernel, kConsumerThreads, kCompactSmem));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, arcv_compact_kernel<kMaxInlineSegs>, kConsumerThreads,
+                                                     kCompactSmem));
     const int k2cap = env_int("ARCV_K2_PER_SM", 2);
     c->k2_grid = c->num_sms * std::max(1, std::min(occ2, k2cap > 0 ? k2cap : 1));
     const int cap = env_int("ARCV_CTAS_PER_SM", 0);

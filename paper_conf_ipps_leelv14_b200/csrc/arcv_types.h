@@ -77,7 +77,7 @@ struct PeerParams {
 };
 
 struct Params {
-    const Seg *segs;          // device table, or nullptr -> inline_segs
+    const Seg *segs;          // device table, or nullptr -> ParamsN::inline_segs
     uint32_t n_segs;
     uint32_t n_acc;
     uint64_t total_tiles;
@@ -109,10 +109,19 @@ struct Params {
     uint32_t flags;
     int xfused;                     // sharded call: K1's CTAs run the exchange after the local result
     PeerParams x;                   // its parameters (xfused only)
-    Seg inline_segs[kMaxInlineSegs];
 };
 
-static_assert(sizeof(Params) <= 4096, "kernel parameters stay within the classic 4 KB limit");
+// The kernels' parameter block: Params plus NSEG inline segments.  The launch
+// cost grows with the parameter bytes (measured: C1 per call 30.0 -> 27.1 us
+// with 1 instead of 16 inline segments), so single-region calls -- the common
+// case -- use NSEG = 1 and batches of up to kMaxInlineSegs regions NSEG = 16;
+// larger batches pass a device table (segs) with NSEG = 1.
+template <int NSEG>
+struct ParamsN : Params {
+    Seg inline_segs[NSEG];
+};
+
+static_assert(sizeof(ParamsN<kMaxInlineSegs>) <= 4096, "kernel parameters stay within the classic 4 KB limit");
 
 struct StageInfo {
     uint64_t tile;        // launch-local tile, ~0 = no more work
