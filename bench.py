@@ -45,6 +45,7 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-configs", action="store_true", help="skip the other BASELINE configs (N = 1)")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no clocks/e2e/cpu)")
     return ap.parse_args()
 
@@ -207,6 +208,72 @@ def cpu_baseline(c4, out_dev, ref_dev):
                       f"contiguous chunks + merge_shards), {reps} repetition(s), {t_all:.1f} s",
             "single_core": {"value": round(gbs_one, 3), "unit": "GB/s", "cores": 1,
                             "sample": f"first 2^24 C4 elements, {reps1} repetition(s), {t_one:.1f} s"}}
+
+
+def other_configs(av, synth, stream, steps=10):
+    """Per-call device time of the other BASELINE configs at N = 1 (C1, C2 A/B, C3 as one
+    batched call, C5), each checked against its generator's closed form.  Arrays smaller than
+    4x L2 get an L2 flush between calls (outside the timed events)."""
+    import torch
+
+    L2 = torch.cuda.get_device_properties(0).L2_cache_size
+    scratch = torch.empty(2 * L2, dtype=torch.uint8, device="cuda")
+    rep = torch.empty(24 * (1 << 20), dtype=torch.uint8, pin_memory=True).numpy().view(av.REPORT_DTYPE)
+    out = {}
+
+    def timed(fn, nbytes, flush):
+        for _ in range(3):
+            res = fn()
+        tot = 0.0
+        for _ in range(steps):
+            if flush:
+                scratch.fill_(1)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            res = fn()
+            e1.record(stream)
+            torch.cuda.synchronize()
+            tot += e0.elapsed_time(e1)
+        us = 1e3 * tot / steps
+        return res, {"per_call_us": round(us, 1), "gbs": round(nbytes / us / 1e3, 1), "l2_flush": flush}
+
+    def idx(r):
+        return [int(i) for i in r.report["index"]]
+
+    c1 = synth.C1()
+    o, r = c1.slice(device="cuda")
+    res, d = timed(av.prepare(o, r, c1.abs_tol, c1.rel_tol, c1.max_report, report=rep), 2 * o.numel() * 4, True)
+    d["parity"] = "ok" if idx(res) == c1.planted() else "FAIL"
+    out["C1 fp32 2^20"] = d
+    del o, r
+    for v in ("A", "B"):
+        c2 = synth.C2(v)
+        o, r = c2.slice(device="cuda")
+        res, d = timed(av.prepare(o, r, c2.abs_tol, c2.rel_tol, c2.max_report, report=rep), 2 * o.numel() * 4,
+                       False)
+        d["parity"] = "ok" if idx(res) == c2.planted() else "FAIL"
+        out[f"C2{v} Jacobi-2D fp32 8192^2"] = d
+        del o, r
+    regs = synth.c3_regions()
+    data = [rg.slice(device="cuda") for rg in regs]
+    nb = sum(2 * o.numel() * o.element_size() for o, _ in data)
+    pb = av.prepare_batch([(o, r, rg.abs_tol, rg.rel_tol, rg.max_report, rg.name) for rg, (o, r) in zip(regs, data)])
+    res, d = timed(pb, nb, True)
+    d["parity"] = "ok" if all(idx(x) == rg.planted()[: rg.max_report] for x, rg in zip(res, regs)) else "FAIL"
+    out["C3 twelve regions, one batched call"] = d
+    del data, pb
+    c5 = synth.C5()
+    o, r = c5.slice(device="cuda")
+    drep = torch.empty(24 * c5.max_report, dtype=torch.uint8, device="cuda")
+    res, d = timed(av.prepare(o, r, 0, 0, c5.max_report, report=drep), 2 * o.numel() * 4, False)
+    first = drep[: 24 * 8].cpu().numpy().view(av.REPORT_DTYPE)
+    d["parity"] = "ok" if (res.n_mismatch == c5.n // 2 and res.n_reported == c5.max_report and
+                           [int(i) for i in first["index"]] == list(range(1, 17, 2))) else "FAIL"
+    d["report"] = "device buffer (2^20 entries)"
+    out["C5 int32 2^30, 50% mismatches"] = d
+    del o, r, drep, scratch
+    torch.cuda.empty_cache()
+    return out
 
 
 # --------------------------------------------------------------------- ours
@@ -379,6 +446,10 @@ def main():
             line["clocks"] = sampler.summary()
         if world == 1 and not args.no_cpu_baseline and not args.profile:
             line["cpu_baseline"] = cpu_baseline(c4, out, ref)
+        if world == 1 and not args.no_configs and not args.profile and n == N_C4:
+            del out, ref
+            torch.cuda.empty_cache()
+            line["other_configs"] = other_configs(av, synth, stream)
         print(json.dumps(line), flush=True)
     av.finalize()
     if world > 1:
