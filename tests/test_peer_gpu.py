@@ -143,3 +143,63 @@ def test_peer_exchange_matches_unsharded_oracle(world, fused, monkeypatch):
                     got = res[0][(name, kind, mr, rep)]
                     assert got[:5] == want[:5], (name, kind, mr, rep, got[:5], want[:5])
                     assert got[5] == want[5], (name, kind, mr, rep)
+
+
+def _stress_worker(rank, world, port, q, calls):
+    sys.path.insert(0, ROOT)
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import paper_conf_ipps_leelv14_b200 as av
+
+        torch.cuda.set_device(0)
+        assert av.init_distributed(transport="peer", max_report_cap=1 << 12) == "peer"
+        regs = [synth.C4(1 << 20), synth.C1()]
+        shards = []
+        for reg in regs:
+            a, b = rank * reg.n // world, (rank + 1) * reg.n // world
+            shards.append(reg.slice(a, b - a, device="cuda"))
+        pinned = torch.empty(24 << 12, dtype=torch.uint8, pin_memory=True).numpy().view(av.REPORT_DTYPE)
+        digest = []
+        for it in range(calls):
+            k = it % 2
+            reg, (o, r) = regs[k], shards[k]
+            mr = (7, 4096, 100)[it % 3]
+            g = av.compare(o, r, reg.abs_tol, reg.rel_tol, mr, report=pinned if it % 5 else None)
+            digest.append((k, mr, g.n_mismatch, g.n_reported,
+                           tuple(int(i) for i in np.asarray(g.report["index"][: g.n_reported]))))
+        av.finalize()
+        q.put((rank, digest, None))
+    except Exception:  # pragma: no cover
+        import traceback
+
+        q.put((rank, None, traceback.format_exc()))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.timeout(600)
+def test_peer_exchange_many_calls():
+    """300 back-to-back sharded calls (world 2, exchange fused into K1): window parities,
+    sequence numbers and the exchange counters stay in step; every call equals the
+    generator's closed form on every rank."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    calls = 300
+    procs = [ctx.Process(target=_stress_worker, args=(r, 2, port, q, calls)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = {}
+    for _ in range(2):
+        rank, digest, err = q.get(timeout=540)
+        assert err is None, f"rank {rank}:\n{err}"
+        res[rank] = digest
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert res[0] == res[1]
+    planted = [synth.C4(1 << 20).planted(), synth.C1().planted()]
+    for k, mr, n_mis, n_rep, head in res[0]:
+        assert n_mis == len(planted[k]) and n_rep == min(n_mis, mr)
+        assert list(head) == planted[k][:n_rep]
