@@ -1085,10 +1085,39 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
     if (warp == 0) {
         if (lane == 0) {
             const uint64_t policy = evict_first_policy();
-            for (uint32_t i = 0;; ++i) {
+            uint64_t t = 0, t_end = 0;  // current run [t, t_end)
+            for (uint32_t i = 0;; ++i, ++t) {
                 const int s = i % S;
                 if (i >= (uint32_t)S) mbar_wait(&empty_bar[s], ((i / S) - 1) & 1);
-                const uint64_t t = atomicAdd(p.ticket, 1ull) - p.ticket_base;
+                if (t >= t_end) {
+#if ARCV_GUIDED
+                  if (p.guided) {
+                    // the counter ends at exactly base + total_tiles: a run that
+                    // crosses the end gives its overshoot back, a run past the
+                    // end all of it (the counter never drops below the end)
+                    // size the run from the counter's current value (a stale
+                    // estimate could hand a long run out near the end)
+                    const uint64_t cur = *(volatile unsigned long long *)p.ticket - p.ticket_base;
+                    const uint64_t rem = p.total_tiles > cur ? p.total_tiles - cur : 0;
+                    uint64_t c = rem / (kGuide * gridDim.x);
+                    c = c < 1 ? 1 : (c > kChunkMax ? kChunkMax : c);
+                    const uint64_t old = atomicAdd(p.ticket, (unsigned long long)c) - p.ticket_base;
+                    if (old >= p.total_tiles) {
+                        atomicAdd(p.ticket, (unsigned long long)(0ull - c));
+                        t = p.total_tiles;
+                    } else {
+                        if (old + c > p.total_tiles)
+                            atomicAdd(p.ticket, (unsigned long long)(0ull - (old + c - p.total_tiles)));
+                        t = old;
+                        t_end = old + c < p.total_tiles ? old + c : p.total_tiles;
+                    }
+                  } else
+#endif
+                  {
+                    t = atomicAdd(p.ticket, 1ull) - p.ticket_base;
+                    t_end = t + 1;
+                  }
+                }
                 if (t >= p.total_tiles) {
                     info[s].tile = ~0ull;
                     mbar_arrive(&full_bar[s]);

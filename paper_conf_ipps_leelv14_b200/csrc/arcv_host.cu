@@ -315,6 +315,7 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
     p.total_tiles = tiles;
     p.ticket = c.counters;
     p.ticket_base = c.ticket_base;
+    p.guided = (ARCV_GUIDED && n_segs > 1) ? 1 : 0;
     p.done = c.counters + 1;
     p.done_base = c.done_base;
     p.tile_cnt = c.tile_cnt;
@@ -373,7 +374,8 @@ int launch_segments(Ctx &c, Seg *segs, uint32_t n_segs, uint32_t acc_lo, uint32_
         : launch_k1_k2<1>(p, segs, n_inl, grid, smem, c.stream, fused || xf, k2, grid2, &c.pdl, &p2);
     if (e != cudaSuccess) return cuda_fail(e, "arcv_stream_kernel / arcv_compact_kernel launch");
     c.launches += k2 ? 2 : 1;
-    c.ticket_base += tiles + grid;
+    if (p.guided) c.ticket_base += tiles;  // runs past the end are given back
+    else c.ticket_base += tiles + grid;    // every producer's last ticket fails
     if (xf) {
         c.peer_done_base += grid;  // every K1 CTA counts once on the exchange counter
         c.x_taken = true;

@@ -149,6 +149,14 @@ def c4shard(lg):
     return f
 
 
+def f32x12():
+    n = 12 * (1 << 22)
+    reg = synth.configs.Region("F", "f32", n, 91, 1e-6, 1e-5, 1024, "f32", n_inject=24)
+    o, r = reg.slice(device="cuda")
+    m = n // 12
+    return batch([(o[k * m:(k + 1) * m], r[k * m:(k + 1) * m], 1e-6, 1e-5, 1024) for k in range(12)])
+
+
 def i32clean():
     reg = synth.configs.Region("I", "i32", 1 << 28, 78, 0, 0, 1 << 20, "i32")
     o, r = reg.slice(device="cuda")
@@ -172,6 +180,7 @@ add("C2A", c2("A"))
 add("C2B", c2("B"))
 add("f32u_2^26", f32u)
 add("C3batch", c3)
+add("f32x12", f32x12)
 add("i32clean_2^28", i32clean)
 add("u8clean_2^30", u8clean)
 add("C4", c4)
