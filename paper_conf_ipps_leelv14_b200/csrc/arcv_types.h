@@ -32,7 +32,10 @@ static_assert(kGroupTiles == kConsumerThreads, "the report phase scans one group
 #ifndef ARCV_GUIDED
 #define ARCV_GUIDED 1
 #endif
-constexpr uint64_t kChunkMax = 8, kGuide = 4;
+#ifndef ARCV_CHUNK_MAX
+#define ARCV_CHUNK_MAX 8
+#endif
+constexpr uint64_t kChunkMax = ARCV_CHUNK_MAX, kGuide = 4;
 
 constexpr uint32_t kFlagProbe = 2u;       // Params.flags: stream only, no predicate (read probe)
 constexpr uint32_t kSegBaseFromAcc = 1u;  // chunk of a streamed region: prefix base = acc count - own total
