@@ -147,6 +147,7 @@ struct ThreadAcc {
 // The fields of the current segment that the per-tile path needs, cached in
 // registers (the Seg table lives in param / global space: generic loads).
 struct SegHot {
+    double (*seed_sh)[2];  // [kConsumerWarps][2] shared scratch: block-wide seeding
     double abs_tol, rel_tol;
     uint64_t max_report, tile_begin, slot_begin, group_begin;
     float at_rd, rt_rd;
@@ -335,6 +336,23 @@ __device__ __forceinline__ uint32_t eval_tile(const uint8_t *so, const uint8_t *
         if (!acc.seeded) {
             seed_bounds<T>(so, sr, off_o, off_r, cnt, ctid, g, acc);
             share_bounds(acc);
+#if !defined(ARCV_BLOCK_SEED) || ARCV_BLOCK_SEED
+            // block-wide: every consumer warp seeds on this same tile (all
+            // threads reset together at a region change), so the 8 warps'
+            // seeded maxima -- folded values, valid bounds -- are pooled:
+            // 8x the samples before the fast filter starts
+            if ((ctid & 31) == 0) {
+                g.seed_sh[ctid >> 5][0] = acc.ma;
+                g.seed_sh[ctid >> 5][1] = acc.rm;
+            }
+            consumer_bar();
+#pragma unroll
+            for (int w = 0; w < kConsumerWarps; ++w) {
+                acc.ma = fmax(acc.ma, g.seed_sh[w][0]);
+                acc.rm = fmax(acc.rm, g.seed_sh[w][1]);
+            }
+            consumer_bar();  // the scratch is reused (flush_acc)
+#endif
         }
         if constexpr (std::is_same<T, float>::value) {
             refresh_bounds(acc, g.at_rd, g.rt_rd, fb);
@@ -1168,6 +1186,7 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
             if (cur >= 0 && slot != g.acc_slot) flush_acc(p.acc, g.acc_slot, g.dtype, acc, ctid, s_red_u, s_red_d);
             cur = (int)si.seg;
             g.load(segs[si.seg]);
+            g.seed_sh = s_red_d;
         }
         const uint8_t *so = smem + (size_t)s * kStageBytes;
         const uint32_t cnt = (p.flags & kFlagProbe) ? 0u : eval_any(so, so + kStageArrayBytes, si, ctid, g, acc);
