@@ -19,6 +19,7 @@ pytestmark = pytest.mark.gpu
 NP = {"f32": np.float32, "f64": np.float64, "i32": np.int32, "i64": np.int64, "u8": np.uint8}
 TD = synth.TORCH_DTYPES
 TILE_ELEMS = {"f32": 4096, "f64": 2048, "i32": 4096, "i64": 2048, "u8": 16384}
+FUZZ_SCALE = int(os.environ.get("ARCV_FUZZ_SCALE", "1"))  # longer seeded fuzz runs on demand
 
 
 def bits(x: float) -> int:
@@ -317,7 +318,7 @@ def test_randomized_fuzz(av, orc):
     rng = np.random.default_rng(20141)
     pinned = torch.empty(24 * 70000, dtype=torch.uint8, pin_memory=True).numpy().view(av.REPORT_DTYPE)
     dev_rep = torch.empty(24 * 70000, dtype=torch.uint8, device="cuda")
-    for it in range(60):
+    for it in range(60 * FUZZ_SCALE):
         dt = ["f32", "f64", "i32", "i64", "u8"][int(rng.integers(5))]
         te = TILE_ELEMS[dt]
         n = int(rng.integers(1, 3000)) * te // 2 + int(rng.integers(0, te))
@@ -338,7 +339,7 @@ def test_randomized_fuzz_batch_and_host(av, orc):
     """Seeded fuzz over batches (1-20 random regions, mixed dtypes and densities, one grid)
     and host-resident inputs (pinned out/ref streamed in chunks: per-chunk report bases)."""
     rng = np.random.default_rng(20142)
-    for it in range(25):
+    for it in range(25 * FUZZ_SCALE):
         regs, exps = [], []
         for k in range(int(rng.integers(1, 21))):
             dt = ["f32", "f64", "i32", "i64", "u8"][int(rng.integers(5))]
