@@ -347,10 +347,13 @@ int arc_verify_shard_merge(const void *gathered_dev, int nranks, uint64_t packet
  * Each rank owns a "window" in its HBM -- 2 x 256 flag words and two packets
  * (call parities) of {32-byte header, max_report_cap entries} -- mapped into
  * every other rank through CUDA IPC (NVLink / NVSwitch peer memory).  A
- * sharded arc_verify_compare with max_report <= max_report_cap then runs
- * local compare -> ONE exchange kernel (publish header + flags with
+ * sharded arc_verify_compare with max_report <= max_report_cap then runs the
+ * local compare and the exchange in ONE kernel (publish header + flags with
  * system-scope release stores into every window, wait for all flags, merge by
- * reading the peers' packets directly) -> one host wait; no NCCL call.
+ * reading the peers' packets directly; a separate exchange kernel for an empty
+ * or host-resident shard) -> one host wait; no NCCL call.  A rank that never
+ * arrives makes the others return ARC_E_CUDA ("peer exchange timed out")
+ * after 60 s instead of hanging.
  * Setup is collective: every rank calls arc_verify_peer_export, the caller
  * all-gathers the 64-byte handles in rank order (e.g. torch.distributed), and
  * every rank calls arc_verify_peer_open.  All ranks must use the same
