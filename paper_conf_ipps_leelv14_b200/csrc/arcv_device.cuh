@@ -784,6 +784,133 @@ __device__ __forceinline__ void grid_barrier(unsigned long long *ctr, unsigned l
     consumer_bar();
 }
 
+// ---- half-block variants: warps 0-3 and 4-7 each handle one tile at once ----
+// (a CTA owning two report tiles processes them concurrently; 128 threads per
+// tile, 8 vectors per thread: element e = ((b / EPV) * 128 + gt) * EPV + b % EPV.
+// Not for u8: 8 x 16 mismatch bits do not fit the 64-bit mask.)
+__device__ __forceinline__ void half_bar(int grp) {
+    asm volatile("bar.sync %0, 128;" ::"r"(2 + grp) : "memory");
+}
+// exclusive scan of two u64 over the 128 threads of half `grp`; totals out
+__device__ __forceinline__ void half_excl_scan2(uint64_t v0, uint64_t v1, uint64_t *s_w, int gt, int grp,
+                                                uint64_t *ex0, uint64_t *ex1, uint64_t *t0, uint64_t *t1) {
+    const int lane = gt & 31, w = gt >> 5;
+    uint64_t a = v0, c = v1;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint64_t ya = __shfl_up_sync(0xffffffffu, a, o);
+        const uint64_t yc = __shfl_up_sync(0xffffffffu, c, o);
+        if (lane >= o) {
+            a += ya;
+            c += yc;
+        }
+    }
+    if (lane == 31) {
+        s_w[2 * w] = a;
+        s_w[2 * w + 1] = c;
+    }
+    half_bar(grp);
+    uint64_t ba = 0, bc = 0, ta = 0, tc = 0;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+        const uint64_t xa = s_w[2 * k], xc = s_w[2 * k + 1];
+        ba += (k < w) ? xa : 0ull;
+        bc += (k < w) ? xc : 0ull;
+        ta += xa;
+        tc += xc;
+    }
+    half_bar(grp);
+    *ex0 = ba + a - v0;
+    *ex1 = bc + c - v1;
+    *t0 = ta;
+    *t1 = tc;
+}
+
+template <typename T>
+__device__ __noinline__ uint64_t mask_tile_half(const uint8_t *so, const uint8_t *sr, uint32_t count, uint32_t off_o,
+                                                uint32_t off_r, int gt, double abs_tol, double rel_tol,
+                                                uint32_t cflags, double minv, double lo, double hi) {
+    constexpr int EPV = 16 / sizeof(T);
+    uint64_t mask = 0;
+#pragma unroll 1
+    for (int b = 0; b < 2 * kVecPerThread * EPV; ++b) {
+        const uint32_t e = (uint32_t)(((b / EPV) * (kConsumerThreads / 2) + gt) * EPV + (b % EPV));
+        if (e >= count) continue;
+        const T xo = *reinterpret_cast<const T *>(so + off_o + e * sizeof(T));
+        const T yr = *reinterpret_cast<const T *>(sr + off_r + e * sizeof(T));
+        const double x = (double)xo, y = (double)yr;
+        if ((cflags & ARC_CHECK_MIN_VALUE) && fabs(y) <= minv) continue;
+        bool mis;
+        if constexpr (std::is_floating_point<T>::value) {
+            const double d = fabs(x - y);
+            const double t = __dadd_rn(abs_tol, __dmul_rn(rel_tol, fabs(y)));
+            mis = !((x == y) | ((x != x) & (y != y)) | ((fabs(y) < CUDART_INF) & (d <= t)));
+        } else {
+            mis = xo != yr;
+        }
+        if (mis && (cflags & ARC_CHECK_VALUE_BOUNDS) && lo <= x && x <= hi) mis = false;
+        mask |= (uint64_t)mis << b;
+    }
+    return mask;
+}
+
+template <typename T>
+__device__ __noinline__ void compact_tile_half(const Seg &g, const StageInfo &si, const uint8_t *so,
+                                               const uint8_t *sr, uint64_t mask, uint64_t excl, uint64_t *s_w,
+                                               int gt, int grp) {
+    constexpr int EPV = 16 / sizeof(T);
+    constexpr int NV = 2 * kVecPerThread;  // 8 vectors: fields 0-3 in p0, 4-7 in p1
+    constexpr uint64_t kGroup = (1ull << EPV) - 1ull;
+    uint64_t p0 = 0, p1 = 0;  // 4 x 16-bit per-k counts each; totals <= 128 * 4
+#pragma unroll
+    for (int k = 0; k < NV; ++k) {
+        const uint64_t c = (uint64_t)__popcll(mask & (kGroup << (k * EPV)));
+        if (k < 4) p0 |= c << (16 * k);
+        else p1 |= c << (16 * (k - 4));
+    }
+    uint64_t ex0, ex1, t0, t1;
+    half_excl_scan2(p0, p1, s_w, gt, grp, &ex0, &ex1, &t0, &t1);
+    arc_mismatch_t *const rep = (excl & kDirectBit) ? g.report_alias : g.report;
+    excl &= ~kDirectBit;
+    uint64_t m = mask;
+    while (m) {
+        const int bpos = __ffsll((long long)m) - 1;
+        m &= m - 1;
+        const int k = bpos / EPV, j = bpos % EPV;
+        uint64_t rank = (uint64_t)__popcll(mask & (((1ull << j) - 1ull) << (k * EPV)));
+        rank += k < 4 ? ((ex0 >> (16 * k)) & 0xffffull) : ((ex1 >> (16 * (k - 4))) & 0xffffull);
+        for (int kk = 0; kk < k; ++kk)
+            rank += kk < 4 ? ((t0 >> (16 * kk)) & 0xffffull) : ((t1 >> (16 * (kk - 4))) & 0xffffull);
+        const uint64_t gi = excl + rank;
+        if (gi < g.max_report) {
+            const uint32_t te = (uint32_t)((k * (kConsumerThreads / 2) + gt) * EPV + j);
+            const T xo = *reinterpret_cast<const T *>(so + si.off_o + te * sizeof(T));
+            const T xr = *reinterpret_cast<const T *>(sr + si.off_r + te * sizeof(T));
+            arc_mismatch_t *dst = rep + gi;
+            dst->index = g.index_base + si.elem_begin + te;
+            dst->out_bits = raw_bits<T>(xo);
+            dst->ref_bits = raw_bits<T>(xr);
+        }
+    }
+}
+
+__device__ __forceinline__ void emit_half_any(const Seg &g, const StageInfo &si, const uint8_t *so, uint64_t excl,
+                                              uint64_t *s_w, int gt, int grp) {
+#define ARCV_HALF(T)                                                                                          \
+    {                                                                                                         \
+        const uint64_t mk = mask_tile_half<T>(so, so + kStageArrayBytes, si.count, si.off_o, si.off_r, gt,     \
+                                              g.abs_tol, g.rel_tol, g.cflags, g.minv, g.lo, g.hi);            \
+        compact_tile_half<T>(g, si, so, so + kStageArrayBytes, mk, excl, s_w, gt, grp);                      \
+    }
+    switch (g.dtype) {
+        case ARC_F32: ARCV_HALF(float) break;
+        case ARC_F64: ARCV_HALF(double) break;
+        case ARC_I32: ARCV_HALF(int32_t) break;
+        default: ARCV_HALF(int64_t) break;
+    }
+#undef ARCV_HALF
+}
+
 __device__ __forceinline__ void compact_any(const Seg &g, const StageInfo &si, const uint8_t *so, const uint8_t *sr,
                                             uint64_t mask, uint64_t excl, uint64_t *s_w, int tid) {
     switch (g.dtype) {
@@ -823,6 +950,7 @@ struct RepShared {
     uint64_t bar[2];
     uint64_t w[kConsumerWarps];
     uint64_t red[kConsumerWarps][4];
+    uint64_t hw[2][8];  // half-block scans (two tiles at once)
     uint64_t owned_pre[kGroupTiles];
     uint32_t owned[kGroupTiles];
     uint32_t n;
@@ -948,6 +1076,37 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
 #pragma unroll
                 for (int c = 0; c < 4; ++c) r[c] += sh.red[w][c];
             if (tid == 0) ARCV_STAMP(1, 3);
+#if !defined(ARCV_HALF_TILES) || ARCV_HALF_TILES
+            if (m == 2 && segs[key[0] >> 40].dtype != ARC_U8 && segs[key[1] >> 40].dtype != ARC_U8) {
+                // the CTA's two tiles at once: warps 0-3 take entry j0 (stage 0),
+                // warps 4-7 entry j0 + 1 (stage 1)
+                const int grp = tid >> 7, gt = tid & 127;
+                const uint64_t kq = grp ? key[1] : key[0];
+                const Seg &g = segs[kq >> 40];
+                const uint64_t seg_tot = grp ? r[3] : r[2];
+                const uint64_t region_cnt = __ldcg(&p.acc[g.acc_slot].count);
+                const uint64_t base = (g.flags & kSegBaseFromAcc) ? region_cnt - seg_tot : 0ull;
+                const uint64_t excl = base + (grp ? r[1] : r[0]);
+                if (gt == 0) p.tile_cnt[g.slot_begin + (kq & kLtMask)] = 0u;  // clean for the next call
+                const bool direct = g.report_alias && !(g.flags & kSegBaseFromAcc) && region_cnt <= kDirectDyn;
+                StageInfo si;
+                uintptr_t ao, ar;
+                uint32_t nbo, nbr;
+                plan_tile(g, kq & kLtMask, si, ao, nbo, ar, nbr);
+                mbar_wait(&sh.bar[grp], phase[grp]);
+                phase[0] ^= 1u;  // both stages' phases complete (each half waits for its own)
+                phase[1] ^= 1u;
+                if (excl < g.max_report)  // uniform within the half
+                    emit_half_any(g, si, smem + (size_t)grp * kStageBytes, excl | (direct ? kDirectBit : 0ull),
+                                  sh.hw[grp], gt, grp);
+                consumer_bar();  // both stages and sh.red are free again
+                if (tid == 0) {
+                    if (j0 + 2 < n_own) issue(__ldcg(p.nz_list + 2 * (b + (j0 + 2) * G)), 0);
+                    if (j0 + 3 < n_own) issue(__ldcg(p.nz_list + 2 * (b + (j0 + 3) * G)), 1);
+                }
+                continue;
+            }
+#endif
             for (uint32_t q = 0; q < m; ++q) {
                 const uint32_t j = j0 + q;
                 const int st = (int)(j & 1);
