@@ -17,7 +17,10 @@ constexpr int kVecPerThread = kTileBytes / 16 / kConsumerThreads;  // 4
 constexpr int kMaxInlineSegs = 16;                 // regions passed as kernel parameters (C3: 12)
 constexpr int kGroupTiles = 256;                    // tiles per group counter
 constexpr int kPoolCap = 2048;                      // report phase, pool path: max listed nonzero tiles
-constexpr uint64_t kDirectDyn = 4096;               // sparse reports: written directly into pinned host memory
+#ifndef ARCV_DIRECT_DYN
+#define ARCV_DIRECT_DYN 4096
+#endif
+constexpr uint64_t kDirectDyn = ARCV_DIRECT_DYN;               // sparse reports: written directly into pinned host memory
 constexpr uint64_t kDirectBit = 1ull << 63;         // report-phase tile prefix flag: entries go to report_alias
 static_assert(kVecPerThread == 4, "packed-scan layout assumes 4 vectors per thread");
 static_assert(kGroupTiles == kConsumerThreads, "the report phase scans one group per block pass");
