@@ -171,7 +171,9 @@ int arc_verify_init(const arc_verify_opts_t *opts);
  * Errors: ARC_E_INVAL (NULL arrays with n > 0, unknown dtype, NaN / negative /
  * infinite tolerance, NULL result, NULL report with max_report > 0, misaligned
  * pointer, device pointer on another device), ARC_E_NOINIT, ARC_E_CUDA,
- * ARC_E_NCCL, ARC_E_NOMEM.
+ * ARC_E_NCCL, ARC_E_NOMEM.  ARC_E_CUDA is also returned when the kernels
+ * finished without publishing this call's results ("completion word
+ * missing"): the library never returns a previous call's numbers as ARC_OK.
  */
 int arc_verify_compare(const void *out, const void *ref, uint64_t n, arc_dtype_t dtype,
                        double abs_tol, double rel_tol, uint64_t max_report,
@@ -282,6 +284,14 @@ int arc_verify_format_result(const char *name, arc_dtype_t dtype, double abs_tol
 /* ABI version (major << 16 | minor). */
 uint32_t arc_verify_version(void);
 
+/* Build description of THIS library (static string, never NULL): the nvcc
+ * flags and -D defines it was compiled with, then the compile-time knobs as
+ * seen by the code itself, e.g. "nvcc: -gencode ... -fmad=false -ftz=false
+ * ...; knobs: ARCV_DIRECT_DYN=4096 ...; defaults=1".  The bit-exact contract
+ * depends on -fmad=false -ftz=false -prec-div=true;
+ * "defaults=0" marks an A/B variant build.  Needs no GPU and no init. */
+const char *arc_verify_build_info(void);
+
 /* ------------------------------------------------------------------------
  * Sharded building blocks (the cross-GPU merge, DESIGN.md sec. 2 step a8).
  * The paper is single-GPU; sharding one large output array across the
@@ -323,10 +333,12 @@ size_t arc_verify_packet_bytes(uint64_t entries);
 
 /*
  * arc_verify_shard_local -- compare one local shard (device pointers) and write
- * its packet to packet_dev (device memory, capacity
- * arc_verify_packet_bytes(max(packet_entries, min(max_report, n))) bytes):
- * header, then the first min(n_mismatch, max_report) local mismatches with
- * LOCAL indices.  Errors as arc_verify_compare.
+ * its packet to packet_dev (device memory of capacity
+ * arc_verify_packet_bytes(packet_entries) bytes, caller-owned): header, then
+ * the first min(n_mismatch, max_report) local mismatches with LOCAL indices.
+ * The kernel may write up to min(max_report, n) entries, so that must not
+ * exceed packet_entries: ARC_E_INVAL otherwise (nothing is launched).  Other
+ * errors as arc_verify_compare.
  */
 int arc_verify_shard_local(const void *out, const void *ref, uint64_t n, arc_dtype_t dtype, double abs_tol,
                            double rel_tol, uint64_t max_report, void *packet_dev, uint64_t packet_entries);

@@ -39,7 +39,7 @@ EXPORTED = [
     "arc_verify_version", "arc_verify_merge_plan", "arc_verify_packet_bytes",
     "arc_verify_shard_local", "arc_verify_shard_merge", "arc_verify_probe_read", "arc_verify_compare_ex",
     "arc_verify_checksum", "arc_verify_selected", "arc_verify_batch_selected", "arc_verify_format_result",
-    "arc_verify_peer_export", "arc_verify_peer_open", "arc_verify_launch_count",
+    "arc_verify_peer_export", "arc_verify_peer_open", "arc_verify_launch_count", "arc_verify_build_info",
 ]
 
 
@@ -107,6 +107,7 @@ def _load() -> ctypes.CDLL:
         "arc_verify_set_timing": (I, [I]),
         "arc_verify_kernel_stats": (I, [ctypes.POINTER(U64), ctypes.POINTER(D), I]),
         "arc_verify_version": (ctypes.c_uint32, []),
+        "arc_verify_build_info": (ctypes.c_char_p, []),
         "arc_verify_merge_plan": (I, [ctypes.POINTER(arc_shard_header_t), I, U64,
                                       ctypes.POINTER(arc_shard_plan_t), ctypes.POINTER(arc_shard_header_t)]),
         "arc_verify_packet_bytes": (SZ, [U64]),
@@ -196,6 +197,10 @@ def arc_verify_kernel_stats(reset: bool = False) -> tuple[int, float]:
 def arc_verify_launch_count() -> int:
     """Kernels the library launched since init (every kernel it owns)."""
     return int(_lib.arc_verify_launch_count())
+
+
+def arc_verify_build_info() -> str:
+    return _lib.arc_verify_build_info().decode()
 
 
 def arc_verify_version() -> int:

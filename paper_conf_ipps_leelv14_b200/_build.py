@@ -10,6 +10,7 @@ No --use_fast_math.
 from __future__ import annotations
 
 import glob
+import json
 import os
 import subprocess
 import sys
@@ -61,18 +62,52 @@ def build(force: bool = False, verbose: bool = False, out: str | None = None, de
         return LIB
     nvcc = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
     tmp = target + f".tmp{os.getpid()}"
-    cmd = [nvcc, *NVCC_FLAGS, *defines, "-I", INCLUDE, "-I", CSRC, "-I", _nccl_include(), "-o", tmp, *sources(),
-           "-ldl"]
-    res = subprocess.run(cmd, capture_output=True, text=True)
-    log = os.path.join(HERE, "build.log")
+    # arc_verify_build_info(): the flags and defines this very library was built
+    # with, compiled into it through a generated header (tests check the shipped
+    # library, not a log a variant build may have overwritten)
+    import tempfile
+
+    gen = tempfile.mkdtemp(prefix="arcv_gen_")
+    info = " ".join(a for a in NVCC_FLAGS if a not in ("-Xptxas", "-v")) + (" " + " ".join(defines) if defines else "")
+    with open(os.path.join(gen, "arcv_build_info.h"), "w") as f:
+        f.write("#pragma once\n#define ARCV_BUILD_FLAGS " + json.dumps(info) + "\n")
+    # one nvcc per translation unit, in parallel (the K1 stage variants are
+    # separate TUs), then one link
+    from concurrent.futures import ThreadPoolExecutor
+
+    objdir = tempfile.mkdtemp(prefix="arcv_obj_")
+    cflags = [a for a in NVCC_FLAGS if a != "-shared"]
+    inc = ["-I", gen, "-I", INCLUDE, "-I", CSRC, "-I", _nccl_include()]
+
+    def compile_one(src):
+        obj = os.path.join(objdir, os.path.basename(src) + ".o")
+        cmd = [nvcc, *cflags, *defines, *inc, "-c", src, "-o", obj]
+        return cmd, obj, subprocess.run(cmd, capture_output=True, text=True)
+
+    with ThreadPoolExecutor(max(1, min(len(sources()), os.cpu_count() or 1))) as ex:
+        results = list(ex.map(compile_one, sources()))
+    link = [nvcc, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-Xcompiler", "-fPIC", "-o", tmp,
+            *[o for _, o, _ in results], "-ldl"]
+    lres = subprocess.run(link, capture_output=True, text=True) if all(r.returncode == 0 for _, _, r in results) \
+        else None
+    # the in-tree log belongs to the in-tree library; a variant logs next to itself
+    log = os.path.join(HERE, "build.log") if out is None else target + ".build.log"
+    text = "".join(" ".join(c) + "\n" + r.stdout + r.stderr for c, _, r in results)
+    if lres is not None:
+        text += " ".join(link) + "\n" + lres.stdout + lres.stderr
     with open(log, "w") as f:
-        f.write(" ".join(cmd) + "\n" + res.stdout + res.stderr)
-    if res.returncode != 0:
-        sys.stderr.write(res.stdout + res.stderr)
+        f.write(text)
+    failed = lres is None or lres.returncode != 0
+    if failed:
+        sys.stderr.write(text[-20000:])
         raise RuntimeError(f"nvcc failed (see {log})")
     if verbose:
-        sys.stderr.write(res.stderr)
+        sys.stderr.write(text)
     os.replace(tmp, target)
+    import shutil
+
+    shutil.rmtree(objdir, ignore_errors=True)
+    shutil.rmtree(gen, ignore_errors=True)
     return target
 
 

@@ -118,7 +118,7 @@ extern "C" int arc_verify_checksum(const void *data, uint64_t bytes, uint64_t *o
         set_error("checksum: device data on the library's device and a non-NULL out are required");
         return ARC_E_INVAL;
     }
-    unsigned long long *acc = c.counters + 5;  // 2 spare u64 counters
+    unsigned long long *acc = c.counters + Ctx::kCtrChecksum;  // its own 2 words (map: arcv_internal.h)
     cudaError_t e = cudaMemsetAsync(acc, 0, 2 * sizeof(unsigned long long), c.stream);
     if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(checksum)");
     if (bytes > 0) {

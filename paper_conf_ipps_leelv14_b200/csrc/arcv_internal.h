@@ -29,8 +29,17 @@ struct Ctx {
     bool own_stream = false;
     cudaStream_t copy_stream = nullptr;
 
-    // monotonic counters: [0] tile tickets, [1] finished CTAs (never reset;
-    // the host tracks each launch's base)
+    // Device counter words (one 64-byte allocation; the map below is the only
+    // place that assigns them -- every user goes through these indices):
+    //   [kCtrTicket]    K1 tile tickets              (monotonic, host-tracked base)
+    //   [kCtrDone]      finished K1/K2 CTAs          (monotonic, host-tracked base)
+    //   [kCtrGbar]      report-phase grid barrier    (monotonic, host-tracked base)
+    //   [kCtrActive]    2 x u32 active-list lengths  (by call parity)
+    //   [kCtrPool]      2 x u32 pool lengths         (by call parity)
+    //   [kCtrPeerDone]  peer-exchange finished blocks (monotonic, peer_done_base)
+    //   [kCtrChecksum]  2 words: checksum sum / xor accumulators (zeroed per call)
+    static constexpr int kCtrTicket = 0, kCtrDone = 1, kCtrGbar = 2, kCtrActive = 3, kCtrPool = 4,
+                         kCtrPeerDone = 5, kCtrChecksum = 6, kCtrWords = 8;
     unsigned long long *counters = nullptr;
     unsigned long long ticket_base = 0, done_base = 0;
 

@@ -1,0 +1,34 @@
+// arcv_k1_s3.cu -- K1 (arcv_stream_kernel) with 3 pipeline stages, min 2 CTAs
+// per SM; one translation unit per stage count (arcv_kernels.h).
+#include <cuda_runtime.h>
+
+#include <vector>
+
+#include "arcv_device.cuh"
+#include "arcv_kernels.h"
+
+namespace arcv {
+
+KernelFnN<1> k1_s3_1() { return arcv_stream_kernel<3, 2, 1>; }
+KernelFnN<kMaxInlineSegs> k1_s3_n() { return arcv_stream_kernel<3, 2, kMaxInlineSegs>; }
+
+// K2: the separate report kernel (used with S = 2 K1s or ARCV_FUSED=0)
+KernelFnN<1> k2_fn_1() { return arcv_compact_kernel<1>; }
+KernelFnN<kMaxInlineSegs> k2_fn_n() { return arcv_compact_kernel<kMaxInlineSegs>; }
+
+// The trace buffer is a __device__ variable of THIS module (the default K1 and
+// K2); other stage counts are not traced.
+int k1_trace_copy(unsigned long long *out, size_t bytes) {
+#if defined(ARCV_TRACE) && ARCV_TRACE
+    if (bytes < sizeof(g_trace)) return -1;
+    if (cudaMemcpyFromSymbol(out, g_trace, sizeof(g_trace)) != cudaSuccess) return -1;
+    std::vector<unsigned long long> zero(sizeof(g_trace) / 8, 0ull);
+    return cudaMemcpyToSymbol(g_trace, zero.data(), sizeof(g_trace)) == cudaSuccess ? 0 : -1;
+#else
+    (void)out;
+    (void)bytes;
+    return -1;
+#endif
+}
+
+}  // namespace arcv

@@ -1,0 +1,15 @@
+// arcv_k1_s4.cu -- K1 (arcv_stream_kernel) with 4 pipeline stages, min 1 CTAs
+// per SM; one translation unit per stage count (arcv_kernels.h).
+#include <cuda_runtime.h>
+
+#include <vector>
+
+#include "arcv_device.cuh"
+#include "arcv_kernels.h"
+
+namespace arcv {
+
+KernelFnN<1> k1_s4_1() { return arcv_stream_kernel<4, 1, 1>; }
+KernelFnN<kMaxInlineSegs> k1_s4_n() { return arcv_stream_kernel<4, 1, kMaxInlineSegs>; }
+
+}  // namespace arcv

@@ -115,7 +115,7 @@ int peer_compare(Ctx &c, const arc_verify_region_t &r, arc_verify_result_t *resu
     // a sparse global report goes straight into a pinned caller buffer
     q.dst_alias = host_report ? static_cast<arc_mismatch_t *>(pinned_device_alias(result->report)) : nullptr;
     q.out = c.peer_out_dev;
-    q.done = c.counters + 5;
+    q.done = c.counters + Ctx::kCtrPeerDone;
     q.done_base = c.peer_done_base;
     q.done_flag = c.flag_dev;
     q.seq = ++c.seq;

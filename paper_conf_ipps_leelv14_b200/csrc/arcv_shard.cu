@@ -357,7 +357,12 @@ int arc_verify_get_unique_id(void *id) {
 int arc_verify_shard_local(const void *out, const void *ref, uint64_t n, arc_dtype_t dtype, double abs_tol,
                            double rel_tol, uint64_t max_report, void *packet_dev, uint64_t packet_entries) {
     if (!g_ctx) return ARC_E_NOINIT;
-    (void)packet_entries;
+    // the local report holds min(max_report, n) entries: it must fit the packet
+    if (std::min<uint64_t>(max_report, n) > packet_entries) {
+        set_error("shard_local: min(max_report, n) = %llu entries exceed the packet capacity %llu",
+                  (unsigned long long)std::min<uint64_t>(max_report, n), (unsigned long long)packet_entries);
+        return ARC_E_INVAL;
+    }
     if (!packet_dev || classify(packet_dev, g_ctx->device) != PK_DEVICE) {
         set_error("packet must be device memory on the library's device");
         return ARC_E_INVAL;

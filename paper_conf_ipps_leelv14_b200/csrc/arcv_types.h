@@ -41,6 +41,7 @@ static_assert(kGroupTiles == kConsumerThreads, "the report phase scans one group
 constexpr uint64_t kChunkMax = ARCV_CHUNK_MAX, kGuide = 4;
 
 constexpr uint32_t kFlagProbe = 2u;       // Params.flags: stream only, no predicate (read probe)
+constexpr uint32_t kEnvFlagMask = 1u | 8u;  // ARCV_FLAGS bits honoured: 1 proxy fence, 8 stream-sync waits
 constexpr uint32_t kSegBaseFromAcc = 1u;  // chunk of a streamed region: prefix base = acc count - own total
 constexpr uint32_t kSegReportHost = 2u;   // `report` is (mapped) host memory (ARCV_WRITER_SYS diagnostic)
 

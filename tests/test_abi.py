@@ -67,12 +67,54 @@ def test_merge_plan_host(lib):
     assert [p[2] for p in plan] == [0, 0, 0]
 
 
-def test_kernel_flags_in_build_log(lib):
-    log = open(os.path.join(os.path.dirname(lib.LIB_PATH), "build.log")).read()
-    first = log.splitlines()[0]
-    for flag in ("-fmad=false", "-ftz=false", "-prec-div=true", "arch=compute_100a,code=sm_100a"):
-        assert flag in first
-    assert "use_fast_math" not in first
+REQUIRED_FLAGS = ("-fmad=false", "-ftz=false", "-prec-div=true", "arch=compute_100a,code=sm_100a")
+
+
+def shipped_build_ok(info: str) -> bool:
+    """The flags the bit-exact contract depends on, no fast
+    math, no -D override, and the code's own knobs at their defaults."""
+    nvcc = info.split("; knobs:")[0]
+    return (all(f in nvcc for f in REQUIRED_FLAGS) and "use_fast_math" not in nvcc
+            and "-fmad=true" not in nvcc and " -D" not in nvcc and info.endswith("defaults=1"))
+
+
+def test_shipped_library_build_flags(lib):
+    """Checked on the loaded library itself (arc_verify_build_info), not on a log."""
+    info = lib.arc_verify_build_info()
+    assert shipped_build_ok(info), info
+
+
+def test_build_info_check_rejects_variants(lib):
+    info = lib.arc_verify_build_info()
+    assert not shipped_build_ok(info.replace("-fmad=false", "-fmad=true"))
+    assert not shipped_build_ok(info.replace("-ftz=false", "-ftz=true"))
+    assert not shipped_build_ok(info.replace("; knobs:", " -DARCV_DIRECT_DYN=65536; knobs:"))
+    assert not shipped_build_ok(info.replace("defaults=1", "defaults=0"))
+    assert not shipped_build_ok(info.replace("-O3", "-O3 --use_fast_math"))
+
+
+@pytest.mark.slow
+def test_variant_build_reports_itself(lib, tmp_path):
+    """A real -D variant build (as tools/ab.py makes) says so in its own build_info,
+    and leaves the in-tree build.log alone."""
+    import importlib.util
+    import subprocess
+    import sys
+
+    spec = importlib.util.spec_from_file_location(
+        "_arcv_build", os.path.join(ROOT, "paper_conf_ipps_leelv14_b200", "_build.py"))
+    b = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(b)
+    log = os.path.join(ROOT, "paper_conf_ipps_leelv14_b200", "build.log")
+    before = open(log).read() if os.path.exists(log) else None
+    so = b.build(out=str(tmp_path / "variant.so"), defines=("-DARCV_DIRECT_DYN=65536",))
+    after = open(log).read() if os.path.exists(log) else None
+    assert before == after
+    code = ("import ctypes,sys; l=ctypes.CDLL(sys.argv[1]); f=l.arc_verify_build_info; "
+            "f.restype=ctypes.c_char_p; print(f().decode())")
+    info = subprocess.run([sys.executable, "-c", code, so], capture_output=True, text=True, check=True).stdout
+    assert "ARCV_DIRECT_DYN=65536" in info and info.strip().endswith("defaults=0")
+    assert not shipped_build_ok(info.strip())
 
 
 def _build_c_example(out_path):

@@ -444,17 +444,21 @@ def test_c4_full_size(av, orc):
 
 
 def test_c5_full_size(av, orc):
+    """C5 at its full size (2^30 int32, 8 GiB read) against the oracle over the WHOLE
+    arrays (all host cores: compare_threads), plus the generator's closed form."""
     c5 = synth.C5()
     out, ref = c5.slice(device="cuda")
-    g = av.compare(out, ref, 0, 0, c5.max_report)
-    # closed form: every odd index mismatches by exactly 1
-    assert g.n_mismatch == 1 << 29 and g.n_reported == 1 << 20
-    assert g.max_abs_err == 1.0 and g.max_rel_err == 0.0
-    # the report is the oracle's on the prefix that holds the first 2^20 mismatches
-    pre = 1 << 21
-    o = orc.compare(out[:pre].cpu().numpy(), ref[:pre].cpu().numpy(), "i32", 0, 0, c5.max_report)
-    assert o.n_mismatch == 1 << 20
-    assert np.array_equal(g.report, o.report)
+    for rep in (None, torch.empty(24 * c5.max_report, dtype=torch.uint8, device="cuda")):
+        g = av.compare(out, ref, 0, 0, c5.max_report, report=rep)
+        # closed form (DESIGN.md sec. 4): every odd index mismatches by exactly 1
+        assert g.n_mismatch == 1 << 29 and g.n_reported == 1 << 20
+        assert g.max_abs_err == 1.0 and g.max_rel_err == 0.0
+        if rep is None:
+            first = g
+    o = orc.compare_threads(out.cpu().numpy(), ref.cpu().numpy(), "i32", 0, 0, c5.max_report)
+    assert_same(first, o, "C5 full")
+    assert_same(g, o, "C5 full, device report")
+    assert np.array_equal(o.report["index"], np.arange(1, 1 << 21, 2, dtype=np.uint64))
 
 
 def test_index_beyond_2_pow_32(av, orc):
@@ -762,3 +766,21 @@ def test_f32_index_beyond_2_pow_32(av):
     assert g.max_abs_err == 1.0 and g.max_rel_err == float("inf")
     del out, ref
     torch.cuda.empty_cache()
+
+
+def test_env_flags_cannot_disable_the_predicate():
+    """ARCV_FLAGS is a diagnostic knob: only bits 1 and 8 are honoured.  Bit 2 is the
+    internal read-probe flag (predicate off); from the environment it must not turn
+    every compare into '0 mismatches, ARC_OK'."""
+    import subprocess
+    import sys
+
+    code = ("import sys; sys.path.insert(0, %r); import synth, paper_conf_ipps_leelv14_b200 as av; "
+            "c1 = synth.C1(); o, r = c1.slice(device='cuda'); av.init(0); "
+            "g = av.compare(o, r, c1.abs_tol, c1.rel_tol, 100); print('COUNT', g.n_mismatch)"
+            % os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    for flags in ("2", "10", "3", "15"):
+        env = dict(os.environ, ARCV_FLAGS=flags)
+        res = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=300, env=env)
+        assert res.returncode == 0, res.stderr[-2000:]
+        assert "COUNT 45" in res.stdout, (flags, res.stdout)

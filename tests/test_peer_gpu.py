@@ -203,3 +203,77 @@ def test_peer_exchange_many_calls():
     for k, mr, n_mis, n_rep, head in res[0]:
         assert n_mis == len(planted[k]) and n_rep == min(n_mis, mr)
         assert list(head) == planted[k][:n_rep]
+
+
+def _checksum_worker(rank, world, port, q):
+    sys.path.insert(0, ROOT)
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    out = []
+    try:
+        import paper_conf_ipps_leelv14_b200 as av
+
+        torch.cuda.set_device(0)
+        assert av.init_distributed(transport="peer", max_report_cap=1 << 12) == "peer"
+        reg = synth.C4(1 << 20)
+        a, b = rank * reg.n // world, (rank + 1) * reg.n // world
+        o, r = reg.slice(a, b - a, device="cuda")
+        pinned = torch.empty(24 << 12, dtype=torch.uint8, pin_memory=True).numpy().view(av.REPORT_DTYPE)
+        for it in range(6):
+            g = av.compare(o, r, reg.abs_tol, reg.rel_tol, 100, report=pinned if it % 2 else None)
+            out.append(("cmp", it, g.n, g.n_mismatch, _bits(g.max_abs_err), _bits(g.max_rel_err), g.n_reported,
+                        np.array(g.report[: g.n_reported]).tobytes()))
+            # the N4 screen between two sharded compares (it used to clobber the
+            # exchange's finished-block counter: every later compare returned the
+            # previous call's summary with ARC_OK)
+            out.append(("sum", it, av.checksum(o), av.checksum(r)))
+        av.finalize()
+        q.put((rank, out, None))
+    except Exception:  # pragma: no cover
+        import traceback
+
+        q.put((rank, out, traceback.format_exc()))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.timeout(600)
+@pytest.mark.parametrize("fused", ["1", "0"])
+def test_checksum_between_sharded_compares(fused, monkeypatch):
+    """compare -> checksum -> compare x 6 on a world-2 peer group: every compare is
+    bit-exact against the unsharded oracle on every rank, every checksum equals the
+    oracle's checksum of the rank's shard."""
+    import oracle
+
+    oracle.build()
+    monkeypatch.setenv("ARCV_FUSED_EXCHANGE", fused)
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_checksum_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = {}
+    for _ in range(world):
+        rank, out, err = q.get(timeout=540)
+        assert err is None, f"rank {rank}:\n{err}"
+        res[rank] = out
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    reg = synth.C4(1 << 20)
+    o, r = reg.slice()
+    e = oracle.compare(o.numpy(), r.numpy(), "f64", reg.abs_tol, reg.rel_tol, 100)
+    want = (e.n, e.n_mismatch, _bits(e.max_abs_err), _bits(e.max_rel_err), e.n_reported,
+            np.ascontiguousarray(e.report).tobytes())
+    for rank in range(world):
+        a, b = rank * reg.n // world, (rank + 1) * reg.n // world
+        sums = (oracle.checksum(o[a:b].numpy()), oracle.checksum(r[a:b].numpy()))
+        cmps = [x for x in res[rank] if x[0] == "cmp"]
+        assert len(cmps) == 6
+        for x in cmps:
+            assert x[2:] == want, (rank, x[1], x[2:7], want[:5])
+        for x in res[rank]:
+            if x[0] == "sum":
+                assert (x[2], x[3]) == sums, (rank, x[1])
