@@ -131,6 +131,25 @@ def _host_cores() -> int:
     return len(os.sched_getaffinity(0))
 
 
+def host_description() -> dict:
+    """lscpu model / sockets / cores of the host the oracle ran on."""
+    import subprocess
+
+    d = {"affinity_threads": _host_cores()}
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        keys = {"Model name": "model", "Socket(s)": "sockets", "Core(s) per socket": "cores_per_socket",
+                "Thread(s) per core": "threads_per_core", "CPU(s)": "cpus", "L3 cache": "l3",
+                "Hypervisor vendor": "hypervisor"}
+        for line in out.splitlines():
+            k, _, v = line.partition(":")
+            if k.strip() in keys:
+                d[keys[k.strip()]] = v.strip()
+    except Exception as e:  # pragma: no cover
+        d["lscpu_error"] = str(e)
+    return d
+
+
 def run_reference(args, rank):
     """The oracle, as it stands, on all host cores (contiguous chunks in host
     threads, merged by the oracle's own merge_shards): each step a bounded
@@ -168,7 +187,8 @@ def run_reference(args, rank):
                    "parallelism": f"{cores} host threads (oracle on contiguous chunks + merge_shards)"},
         "parity": "ok" if list(res.report["index"]) == planted[: c4.max_report] else "FAIL",
         "cpu_baseline": {"value": round(gbs, 3), "unit": "GB/s", "cores": cores, "kind": "oracle",
-                         "sample": f"first 2^24 of 2^29 C4 elements, {args.steps} steps"},
+                         "sample": f"first 2^24 of 2^29 C4 elements, {args.steps} steps",
+                         "host": host_description()},
         "e2e": {"value": round(gbs, 3), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -204,6 +224,7 @@ def cpu_baseline(c4, out_dev, ref_dev):
     reps1, t_one = timed(lambda: oracle.compare(o[:small], r[:small], "f64", c4.abs_tol, c4.rel_tol, c4.max_report))
     gbs_one = 2 * small * ES * reps1 / t_one / 1e9
     return {"value": round(gbs_all, 3), "unit": "GB/s", "cores": cores, "kind": "oracle",
+            "host": host_description(),
             "sample": f"first 2^26 of the 2^29 C4 elements (fp64) on {cores} host threads (oracle on "
                       f"contiguous chunks + merge_shards), {reps} repetition(s), {t_all:.1f} s",
             "single_core": {"value": round(gbs_one, 3), "unit": "GB/s", "cores": 1,
@@ -436,6 +457,10 @@ def main():
                          "frac": round(achieved / peak, 4),
                          # the committed ncu capture is of this exact launch only at N = 1 on C4
                          "traffic": ncu_traffic() if (world == 1 and n == N_C4) else None,
+                         "traffic_source": ("committed ncu --set full capture of this launch "
+                                            "(profiles/ncu_summary.json: dram__bytes_read.sum + "
+                                            "dram__bytes_write.sum), not measured in this run"
+                                            if (world == 1 and n == N_C4) else None),
                          "kernel": "arcv_stream_kernel (report phase fused in its tail)", "kernel_ms_avg": round(kern_avg_ms, 4),
                          "algorithmic_bytes_per_launch": local_bytes, "peak_source": peak_src,
                          "read_probe_gbs": round(probe, 1) if probe else None,

@@ -385,6 +385,16 @@ int arc_verify_peer_export(uint64_t max_report_cap, void *handle);
  * be mapped, e.g. no P2P between the devices; the NCCL path stays in use). */
 int arc_verify_peer_open(const void *handles);
 
+/* Bytes this rank's exchanges have read from OTHER ranks' windows since the
+ * last reset: bytes[0] = report entries pulled from the contributing ranks'
+ * packets, bytes[1] = entries read from a forwarding neighbour (ring mode,
+ * p >= 3 and a global report of >= 2^17 entries travels
+ * owner -> owner+1 -> ... in 384 KB chunks, so no window is read more than
+ * once per call).  Measured by the exchange kernels (one atomic per warp).
+ * reset != 0 clears the counters.  Synchronises the library's stream.
+ * Errors: ARC_E_NOINIT, ARC_E_INVAL (bytes NULL), ARC_E_CUDA. */
+int arc_verify_peer_stats(uint64_t *bytes, int reset);
+
 #ifdef __cplusplus
 }
 #endif

@@ -40,6 +40,7 @@ EXPORTED = [
     "arc_verify_shard_local", "arc_verify_shard_merge", "arc_verify_probe_read", "arc_verify_compare_ex",
     "arc_verify_checksum", "arc_verify_selected", "arc_verify_batch_selected", "arc_verify_format_result",
     "arc_verify_peer_export", "arc_verify_peer_open", "arc_verify_launch_count", "arc_verify_build_info",
+    "arc_verify_peer_stats",
 ]
 
 
@@ -108,6 +109,7 @@ def _load() -> ctypes.CDLL:
         "arc_verify_kernel_stats": (I, [ctypes.POINTER(U64), ctypes.POINTER(D), I]),
         "arc_verify_version": (ctypes.c_uint32, []),
         "arc_verify_build_info": (ctypes.c_char_p, []),
+        "arc_verify_peer_stats": (I, [ctypes.POINTER(U64), I]),
         "arc_verify_merge_plan": (I, [ctypes.POINTER(arc_shard_header_t), I, U64,
                                       ctypes.POINTER(arc_shard_plan_t), ctypes.POINTER(arc_shard_header_t)]),
         "arc_verify_packet_bytes": (SZ, [U64]),
@@ -237,6 +239,13 @@ def arc_verify_peer_export(max_report_cap: int) -> bytes:
     buf = ctypes.create_string_buffer(64)
     _check(_lib.arc_verify_peer_export(max_report_cap, buf), "arc_verify_peer_export")
     return buf.raw
+
+
+def arc_verify_peer_stats(reset: bool = False) -> tuple[int, int]:
+    """(bytes pulled from owners' packets, bytes read from a forwarding neighbour)."""
+    b = (ctypes.c_uint64 * 2)()
+    _check(_lib.arc_verify_peer_stats(b, int(reset)), "arc_verify_peer_stats")
+    return int(b[0]), int(b[1])
 
 
 def arc_verify_peer_open(handles: Sequence[bytes]) -> None:

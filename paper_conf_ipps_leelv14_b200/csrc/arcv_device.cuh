@@ -594,15 +594,23 @@ __device__ __forceinline__ bool last_cta(const Params &p, int tid, int nthreads,
     return *s_last != 0;
 }
 
-__device__ __forceinline__ void publish(const Params &p, int tid, int nthreads) {
+// `fenced` = false for launches that wrote no report entry to host memory (a
+// clean or count-only call): the slots validate themselves (slot_tag), so the
+// completion word needs no system fence -- one PCIe round trip (~3 us) less
+// in the last CTA.  With entries written over PCIe the cumulative system fence
+// orders them (and the slots) before the word.
+__device__ __forceinline__ void publish(const Params &p, int tid, int nthreads, bool fenced = true) {
     {
         fence_gpu();
+        // the report phase's path (the host re-applies direct_route with it)
+        const unsigned long long route =
+            (p.k2 && *(volatile uint32_t *)p.nz_cnt <= (uint32_t)kPoolCap) ? kRoutePool : 0ull;
         for (uint32_t k = tid; k < p.n_acc; k += nthreads) {
             Acc a;
             a.count = __ldcg(&p.acc[k].count);
             a.max_abs_bits = __ldcg(&p.acc[k].max_abs_bits);
             a.max_rel_bits = __ldcg(&p.acc[k].max_rel_bits);
-            a.pad = 0;
+            a.pad = slot_tag(p.seq, route, a.count, a.max_abs_bits, a.max_rel_bits);
             p.result[k] = a;
             if (p.mirror) p.mirror[k] = a;
             p.acc[k].count = 0;
@@ -612,7 +620,7 @@ __device__ __forceinline__ void publish(const Params &p, int tid, int nthreads) 
         if (p.done_flag) {
             if (nthreads == kConsumerThreads) consumer_bar(); else __syncthreads();
             if (tid == 0) {
-                fence_sys();
+                if (fenced) fence_sys();
                 *(volatile unsigned long long *)p.done_flag = p.seq;
             }
         }
@@ -632,8 +640,11 @@ __device__ __forceinline__ void finalize_launch(const Params &p, int tid, int nt
 // stage memory.
 __device__ __forceinline__ void exchange_tail(const Params &p, int tid, bool leader, uint8_t *smem) {
     if (leader && tid == 0) {
-        const Acc a = p.mirror[0];  // this thread wrote it in publish()
-        peer_publish_header(p.x, a.count, a.max_abs_bits, a.max_rel_bits);
+        // written by publish() in this CTA or (clean fused call) in the CTA that
+        // arrived last at the grid barrier, released before its done count
+        fence_gpu();  // acquire side of that release (the done count was observed above)
+        const Acc *m = p.mirror;
+        peer_publish_header(p.x, __ldcg(&m->count), __ldcg(&m->max_abs_bits), __ldcg(&m->max_rel_bits));
     }
     peer_exchange_body(p.x, tid, *reinterpret_cast<ExShared *>(smem));
 }
@@ -666,9 +677,16 @@ __device__ __forceinline__ uint64_t block_excl_scan(uint64_t v, uint64_t *s_w, u
 
 // Writes this tile's mismatches with global report rank excl + in-tile rank,
 // for ranks < max_report.  In-tile order = element index order = (k, tid, j).
+// `obuf` non-null (a dense tile going to pinned host memory): only the tile's
+// in-tile ranks [rlo, rhi) are written, in rounds of kOutEntries entries staged
+// in shared memory and stored as consecutive 8-byte words (one warp store =
+// 256 contiguous bytes, i.e. full PCIe write packets instead of 24-byte
+// scatter).  Called by all 256 consumer threads (it synchronises them).
+constexpr int kOutEntries = 1024;
 template <typename T>
 __device__ __noinline__ void compact_tile(const Seg &g, const StageInfo &si, const uint8_t *so, const uint8_t *sr,
-                                          uint64_t mask, uint64_t excl, uint64_t *s_w, int tid) {
+                                          uint64_t mask, uint64_t excl, uint64_t *s_w, int tid, uint64_t rlo,
+                                          uint64_t rhi, arc_mismatch_t *obuf) {
     constexpr int EPV = 16 / sizeof(T);
     constexpr uint64_t kGroup = EPV == 64 ? ~0ull : ((1ull << EPV) - 1ull);
     uint64_t packed = 0;  // 4 x 16-bit per-k counts; field totals <= 4096 (no carries)
@@ -679,6 +697,37 @@ __device__ __noinline__ void compact_tile(const Seg &g, const StageInfo &si, con
     const uint64_t ex = block_excl_scan(packed, s_w, &total, tid);
     arc_mismatch_t *const rep = (excl & kDirectBit) ? g.report_alias : g.report;
     excl &= ~kDirectBit;
+    if (obuf) {
+        const uint64_t lim = g.max_report > excl ? g.max_report - excl : 0ull;  // reported ranks < lim
+        const uint64_t hi = rhi < lim ? rhi : lim;
+        for (uint64_t r0 = rlo; r0 < hi; r0 += kOutEntries) {  // uniform
+            const uint64_t r1 = r0 + kOutEntries < hi ? r0 + kOutEntries : hi;
+            uint64_t m = mask;
+            while (m) {
+                const int b = __ffsll((long long)m) - 1;
+                m &= m - 1;
+                const int k = b / EPV, j = b % EPV;
+                uint64_t rank = ((ex >> (16 * k)) & 0xffffull) +
+                                (uint64_t)__popcll(mask & (((1ull << j) - 1ull) << (k * EPV)));
+                for (int kk = 0; kk < k; ++kk) rank += (total >> (16 * kk)) & 0xffffull;
+                if (rank >= r0 && rank < r1) {
+                    const uint32_t te = (uint32_t)((k * kConsumerThreads + tid) * EPV + j);
+                    arc_mismatch_t e;
+                    e.index = g.index_base + si.elem_begin + te;
+                    e.out_bits = raw_bits<T>(*reinterpret_cast<const T *>(so + si.off_o + te * sizeof(T)));
+                    e.ref_bits = raw_bits<T>(*reinterpret_cast<const T *>(sr + si.off_r + te * sizeof(T)));
+                    obuf[rank - r0] = e;
+                }
+            }
+            consumer_bar();
+            const uint64_t nw = 3 * (r1 - r0);
+            const unsigned long long *src = reinterpret_cast<const unsigned long long *>(obuf);
+            unsigned long long *dst = reinterpret_cast<unsigned long long *>(rep + excl + r0);
+            for (uint64_t w = tid; w < nw; w += kConsumerThreads) dst[w] = src[w];
+            consumer_bar();  // obuf is reused
+        }
+        return;
+    }
     uint64_t m = mask;
     while (m) {
         const int b = __ffsll((long long)m) - 1;
@@ -912,13 +961,14 @@ __device__ __forceinline__ void emit_half_any(const Seg &g, const StageInfo &si,
 }
 
 __device__ __forceinline__ void compact_any(const Seg &g, const StageInfo &si, const uint8_t *so, const uint8_t *sr,
-                                            uint64_t mask, uint64_t excl, uint64_t *s_w, int tid) {
+                                            uint64_t mask, uint64_t excl, uint64_t *s_w, int tid, uint64_t rlo,
+                                            uint64_t rhi, arc_mismatch_t *obuf) {
     switch (g.dtype) {
-        case ARC_F32: compact_tile<float>(g, si, so, sr, mask, excl, s_w, tid); break;
-        case ARC_F64: compact_tile<double>(g, si, so, sr, mask, excl, s_w, tid); break;
-        case ARC_I32: compact_tile<int32_t>(g, si, so, sr, mask, excl, s_w, tid); break;
-        case ARC_I64: compact_tile<int64_t>(g, si, so, sr, mask, excl, s_w, tid); break;
-        default: compact_tile<uint8_t>(g, si, so, sr, mask, excl, s_w, tid); break;
+        case ARC_F32: compact_tile<float>(g, si, so, sr, mask, excl, s_w, tid, rlo, rhi, obuf); break;
+        case ARC_F64: compact_tile<double>(g, si, so, sr, mask, excl, s_w, tid, rlo, rhi, obuf); break;
+        case ARC_I32: compact_tile<int32_t>(g, si, so, sr, mask, excl, s_w, tid, rlo, rhi, obuf); break;
+        case ARC_I64: compact_tile<int64_t>(g, si, so, sr, mask, excl, s_w, tid, rlo, rhi, obuf); break;
+        default: compact_tile<uint8_t>(g, si, so, sr, mask, excl, s_w, tid, rlo, rhi, obuf); break;
     }
 }
 
@@ -957,7 +1007,8 @@ struct RepShared {
     int last;
     int wrote;  // this CTA wrote report entries to pinned host memory
 };
-constexpr int kReportSmem = 2 * kStageBytes + (int)sizeof(RepShared);
+// [stage 0][stage 1][RepShared][out buffer: kOutEntries entries]
+constexpr int kReportSmem = 2 * kStageBytes + (int)sizeof(RepShared) + kOutEntries * (int)sizeof(arc_mismatch_t);
 
 __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, uint8_t *smem, int tid,
                                              unsigned long long done_base, bool k1_published_if_empty) {
@@ -972,7 +1023,7 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
     consumer_bar();
     const uint64_t policy = evict_first_policy();
     constexpr uint64_t kLtMask = (1ull << 40) - 1;
-    uint32_t phase[2] = {0u, 0u};
+    uint32_t phase = 0u;  // bit st: the parity stage st's barrier waits for next (no local array)
     auto issue = [&](uint64_t key, int st) {
         const Seg &g = segs[key >> 40];
         StageInfo si;
@@ -986,26 +1037,37 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
     };
     // wait for tile `key` in stage st, write its entries from report rank excl.
     // A region with a report_alias (pinned host memory, the caller's or the
-    // library's staging for a pageable buffer) and at most kDirectDyn
-    // mismatches in total -- K1's final count; the host applies the same rule
-    // to n_mismatch -- gets its entries written there directly over PCIe.
-    auto emit = [&](uint64_t key, uint64_t excl, int st, bool stamp = false) {
+    // library's staging for a pageable buffer) gets its entries written there
+    // directly over PCIe when direct_route() holds -- K1's final count and the
+    // path taken decide it; the host applies the same rule to the published
+    // slot.  `tc` = the tile's count (pool path; 0 if unknown), `part` / `S`:
+    // this CTA writes in-tile ranks [part * ceil(tc / S), ...) only (a dense
+    // tile split across S CTAs); split or dense direct tiles go through the
+    // shared-memory out buffer (coalesced stores).
+    arc_mismatch_t *const obuf = reinterpret_cast<arc_mismatch_t *>(smem + 2 * kStageBytes + sizeof(RepShared));
+    auto emit = [&](uint64_t key, uint64_t excl, int st, bool pool, uint64_t tc, uint32_t part, uint32_t S,
+                    bool stamp = false) {
         const Seg &g = segs[key >> 40];
-        const bool direct = g.report_alias && !(g.flags & kSegBaseFromAcc) &&
-                            __ldcg(&p.acc[g.acc_slot].count) <= kDirectDyn;
+        const bool direct = direct_route(g.report_alias != nullptr, g.flags, __ldcg(&p.acc[g.acc_slot].count),
+                                         g.max_report, g.alias_cap, pool);
         StageInfo si;
         uintptr_t ao, ar;
         uint32_t nbo, nbr;
         plan_tile(g, key & kLtMask, si, ao, nbo, ar, nbr);
-        mbar_wait(&sh.bar[st], phase[st]);
-        phase[st] ^= 1u;
+        mbar_wait(&sh.bar[st], (phase >> st) & 1u);
+        phase ^= 1u << st;
         if (tid == 0 && stamp) ARCV_STAMP(1, 4);
         if (excl < g.max_report) {  // uniform
             if ((direct || (g.flags & kSegReportHost)) && tid == 0) sh.wrote = 1;
             const uint8_t *so = smem + (size_t)st * kStageBytes;
             const uint64_t mask = mask_any(so, so + kStageArrayBytes, si, tid, g);
             if (tid == 0 && stamp) ARCV_STAMP(1, 5);
-            compact_any(g, si, so, so + kStageArrayBytes, mask, excl | (direct ? kDirectBit : 0ull), sh.w, tid);
+            const bool staged = S > 1 || (direct && tc > kStagedMin);
+            const uint64_t per = (tc + S - 1) / S;
+            const uint64_t rlo = staged ? (uint64_t)part * per : 0ull;
+            const uint64_t rhi = staged ? (rlo + per < tc ? rlo + per : tc) : ~0ull;
+            compact_any(g, si, so, so + kStageArrayBytes, mask, excl | (direct ? kDirectBit : 0ull), sh.w, tid,
+                        rlo, rhi, staged ? obuf : nullptr);
         }
         consumer_bar();  // stage `st` and sh.w are reused
         if (tid == 0 && stamp) ARCV_STAMP(1, 2);
@@ -1017,16 +1079,29 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
         // ------------------------------------------------------ pool path
         // arrive on the grid-barrier counter without waiting (host base += grid)
         if (tid == 0) atomicAdd(p.gbar, 1ull);
+        // few listed tiles that are dense on average (> kStagedMin mismatches per
+        // tile): each is split across S CTAs, so a dense tile's entries are
+        // written by S SMs; work item i = pool entry i / S, part i % S.  Every
+        // CTA derives the same S from the final counts.
+        uint32_t S = 1u;
+        if (n_nz > 0 && 2 * n_nz <= G && p.n_segs <= (uint32_t)kMaxInlineSegs) {
+            uint64_t tot_cnt = 0;
+            for (uint32_t sgi = 0; sgi < p.n_segs; ++sgi)
+                if (segs[sgi].max_report) tot_cnt += __ldcg(&p.acc[segs[sgi].acc_slot].count);
+            if (tot_cnt > (uint64_t)n_nz * kStagedMin) S = min(kSplitMax, G / n_nz);
+        }
+        const uint32_t n_items = n_nz * S;
 #if defined(ARCV_TAIL_REPS)
       // diagnostic: run the (idempotent) pool path again, stamps from the last run
       for (int rep_ = 0; rep_ < ARCV_TAIL_REPS; ++rep_) {
         consumer_bar();
         if (tid == 0) ARCV_STAMP(1, 8);
 #endif
-        const uint32_t n_own = n_nz > b ? (n_nz - b + G - 1) / G : 0u;
+        const uint32_t n_own = n_items > b ? (n_items - b + G - 1) / G : 0u;
+        auto entry_of = [&](uint32_t j) { return (b + j * G) / S; };  // my j-th item's pool entry
         if (tid == 0 && n_own > 0) {  // both key loads in flight before the first issue
-            const uint64_t k0 = __ldcg(p.nz_list + 2 * b);
-            const uint64_t k1 = n_own > 1 ? __ldcg(p.nz_list + 2 * (b + G)) : 0ull;
+            const uint64_t k0 = __ldcg(p.nz_list + 2 * entry_of(0));
+            const uint64_t k1 = n_own > 1 ? __ldcg(p.nz_list + 2 * entry_of(1)) : 0ull;
             issue(k0, 0);
             if (n_own > 1) issue(k1, 1);
         }
@@ -1047,9 +1122,20 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
 #endif
         for (uint32_t j0 = 0; j0 < n_own; j0 += 2) {
             const uint32_t m = n_own - j0 < 2u ? n_own - j0 : 2u;
-            uint64_t key[2], pre[2] = {0, 0}, tot[2] = {0, 0};
-            key[0] = __ldcg(p.nz_list + 2 * (b + j0 * G));
-            key[1] = m > 1 ? __ldcg(p.nz_list + 2 * (b + (j0 + 1) * G)) : ~0ull - 1;
+            uint64_t key[2], tcn[2] = {0, 0}, pre[2] = {0, 0}, tot[2] = {0, 0};
+            uint32_t part[2] = {0, 0};
+#pragma unroll
+            for (int q = 0; q < 2; ++q) {
+                if ((uint32_t)q < m) {
+                    const uint32_t e = entry_of(j0 + q);
+                    const ulonglong2 kv = __ldcg(reinterpret_cast<const ulonglong2 *>(p.nz_list) + e);
+                    key[q] = kv.x;
+                    tcn[q] = kv.y;
+                    part[q] = (b + (j0 + q) * G) % S;
+                } else {
+                    key[q] = ~0ull - 1;
+                }
+            }
 #pragma unroll
             for (int u = 0; u < kPer; ++u)
 #pragma unroll
@@ -1077,7 +1163,18 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
                 for (int c = 0; c < 4; ++c) r[c] += sh.red[w][c];
             if (tid == 0) ARCV_STAMP(1, 3);
 #if !defined(ARCV_HALF_TILES) || ARCV_HALF_TILES
-            if (m == 2 && segs[key[0] >> 40].dtype != ARC_U8 && segs[key[1] >> 40].dtype != ARC_U8) {
+            bool half = m == 2 && S == 1 && segs[key[0] >> 40].dtype != ARC_U8 && segs[key[1] >> 40].dtype != ARC_U8;
+            if (half) {  // not for dense tiles going straight to pinned memory (staged writes)
+#pragma unroll
+                for (int q = 0; q < 2; ++q) {
+                    const Seg &gq = segs[key[q] >> 40];
+                    if (tcn[q] > kStagedMin &&
+                        direct_route(gq.report_alias != nullptr, gq.flags, __ldcg(&p.acc[gq.acc_slot].count),
+                                     gq.max_report, gq.alias_cap, true))
+                        half = false;
+                }
+            }
+            if (half) {
                 // the CTA's two tiles at once: warps 0-3 take entry j0 (stage 0),
                 // warps 4-7 entry j0 + 1 (stage 1)
                 const int grp = tid >> 7, gt = tid & 127;
@@ -1088,36 +1185,37 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
                 const uint64_t base = (g.flags & kSegBaseFromAcc) ? region_cnt - seg_tot : 0ull;
                 const uint64_t excl = base + (grp ? r[1] : r[0]);
                 if (gt == 0) p.tile_cnt[g.slot_begin + (kq & kLtMask)] = 0u;  // clean for the next call
-                const bool direct = g.report_alias && !(g.flags & kSegBaseFromAcc) && region_cnt <= kDirectDyn;
+                const bool direct = direct_route(g.report_alias != nullptr, g.flags, region_cnt, g.max_report,
+                                                 g.alias_cap, true);
                 StageInfo si;
                 uintptr_t ao, ar;
                 uint32_t nbo, nbr;
                 plan_tile(g, kq & kLtMask, si, ao, nbo, ar, nbr);
-                mbar_wait(&sh.bar[grp], phase[grp]);
-                phase[0] ^= 1u;  // both stages' phases complete (each half waits for its own)
-                phase[1] ^= 1u;
+                mbar_wait(&sh.bar[grp], (phase >> grp) & 1u);
+                phase ^= 3u;  // both stages' phases complete (each half waits for its own)
                 if (excl < g.max_report)  // uniform within the half
                     emit_half_any(g, si, smem + (size_t)grp * kStageBytes, excl | (direct ? kDirectBit : 0ull),
                                   sh.hw[grp], gt, grp);
                 consumer_bar();  // both stages and sh.red are free again
                 if (tid == 0) {
-                    if (j0 + 2 < n_own) issue(__ldcg(p.nz_list + 2 * (b + (j0 + 2) * G)), 0);
-                    if (j0 + 3 < n_own) issue(__ldcg(p.nz_list + 2 * (b + (j0 + 3) * G)), 1);
+                    if (j0 + 2 < n_own) issue(__ldcg(p.nz_list + 2 * entry_of(j0 + 2)), 0);
+                    if (j0 + 3 < n_own) issue(__ldcg(p.nz_list + 2 * entry_of(j0 + 3)), 1);
                 }
                 continue;
             }
 #endif
-            for (uint32_t q = 0; q < m; ++q) {
+#pragma unroll
+            for (int q = 0; q < 2; ++q) {
+                if ((uint32_t)q >= m) break;
                 const uint32_t j = j0 + q;
-                const int st = (int)(j & 1);
                 const Seg &g = segs[key[q] >> 40];
                 const uint64_t seg_tot = r[2 + q];
                 uint64_t base = 0;
                 if (g.flags & kSegBaseFromAcc) base = __ldcg(&p.acc[g.acc_slot].count) - seg_tot;
-                if (tid == 0) p.tile_cnt[g.slot_begin + (key[q] & kLtMask)] = 0u;  // clean for the next call
-                emit(key[q], base + r[q], st, j == 0);  // ends with a barrier: sh.red free again
+                if (tid == 0 && part[q] == 0) p.tile_cnt[g.slot_begin + (key[q] & kLtMask)] = 0u;  // clean
+                emit(key[q], base + r[q], q, true, tcn[q], part[q], S, j == 0);  // ends with a barrier
                 if (tid == 0 && j == 1) ARCV_STAMP(1, 10);
-                if (tid == 0 && j + 2 < n_own) issue(__ldcg(p.nz_list + 2 * (b + (j + 2) * G)), st);
+                if (tid == 0 && j + 2 < n_own) issue(__ldcg(p.nz_list + 2 * entry_of(j + 2)), q);
             }
         }
         if (tid == 0) ARCV_STAMP(1, 6);
@@ -1190,7 +1288,7 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
             if (j + 1 < mine && tid == 0) issue(__ldcg(p.active + 2 * (b + (j + 1) * G)), st ^ 1);  // prefetch
             const uint64_t key = __ldcg(p.active + 2 * (b + j * G));
             const uint64_t excl = __ldcg(p.active + 2 * (b + j * G) + 1);
-            emit(key, excl, st);
+            emit(key, excl, st, false, 0, 0, 1);
         }
     }
     // Report entries in pinned host memory need no system-scope fence here:
@@ -1338,6 +1436,7 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
     for (uint32_t i = 0;; ++i) {
         const int s = i % S;
         mbar_wait(&full_bar[s], (i / S) & 1);
+        if (ctid == 0 && i == 0) ARCV_STAMP(0, 4);
         const StageInfo si = info[s];
         if (si.tile == ~0ull) break;
         if ((int)si.seg != cur) {
@@ -1350,6 +1449,7 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
         const uint8_t *so = smem + (size_t)s * kStageBytes;
         const uint32_t cnt = (p.flags & kFlagProbe) ? 0u : eval_any(so, so + kStageArrayBytes, si, ctid, g, acc);
         acc.count += cnt;
+        if (ctid == 0 && i == 0) ARCV_STAMP(0, 5);
         if (g.max_report != 0) {
             // Per-tile count for the report phase: warps fold their counts into the stage's
             // shared word (arrivals << 24 | count); the last warp publishes the
@@ -1405,11 +1505,19 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
             if (ctid == 0) {
                 ARCV_STAMP(1, 0);
                 fence_gpu();
-                atomicAdd(p.done, 1ull);
-                while (ld_acquire_u64(p.done) - p.done_base < (unsigned long long)gridDim.x) __nanosleep(32);
+                const unsigned long long prev = atomicAdd(p.done, 1ull);
+                s_last = (prev - p.done_base) == (unsigned long long)(gridDim.x - 1);
+                if (!s_last)
+                    while (ld_acquire_u64(p.done) - p.done_base < (unsigned long long)gridDim.x) __nanosleep(32);
             }
             consumer_bar();
-            report_phase(p, segs, smem, ctid, p.done_base + gridDim.x, false);
+            // The CTA that arrives last has seen every count: with no tile to
+            // report (the common, clean call) the results are final now, so it
+            // publishes at once instead of after the report phase's own round
+            // (which then only keeps the counter contract).
+            if (s_last && p.finalize && *(volatile uint32_t *)p.nz_cnt == 0u)
+                publish(p, ctid, kConsumerThreads, false);  // no report entry written anywhere
+            report_phase(p, segs, smem, ctid, p.done_base + gridDim.x, true);
             return;
         }
     }
@@ -1418,7 +1526,8 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
     // here while K2 -- then a no-op -- runs in the background.
     if ((p.finalize || p.k2) && last_cta(p, ctid, kConsumerThreads, &s_last, false, p.done_base)) {
         fence_gpu();
-        if (p.finalize && (!p.k2 || *(volatile uint32_t *)p.nz_cnt == 0u)) publish(p, ctid, kConsumerThreads);
+        if (p.finalize && (!p.k2 || *(volatile uint32_t *)p.nz_cnt == 0u))
+            publish(p, ctid, kConsumerThreads, false);  // count-only / clean: no report entry written
     }
     if (p.xfused) exchange_tail(p, ctid, s_last != 0, smem);  // count-only sharded call (no K2 then)
     if (ctid == 0) ARCV_STAMP(0, 3);

@@ -99,6 +99,9 @@ struct Ctx {
     unsigned long long coll_seq = 0;   // collective calls made (flag value of the last)
     unsigned long long peer_done_base = 0;
     arc_shard_header_t *peer_out_host = nullptr, *peer_out_dev = nullptr;  // mapped [2]: global, status
+    uint32_t *ring_cnt = nullptr;      // [2][ring_cnt_n] ring-forwarding chunk counters (zero at export)
+    uint64_t ring_cnt_n = 0;
+    unsigned long long *peer_stats = nullptr;  // [2] bytes read from peer windows (owners / forwarders)
 };
 
 extern Ctx *g_ctx;

@@ -74,6 +74,11 @@ void peer_finalize(Ctx &c) {
     if (c.win_table) cudaFree(c.win_table);
     if (c.mirror) cudaFree(c.mirror);
     if (c.peer_out_host) cudaFreeHost(c.peer_out_host);
+    if (c.ring_cnt) cudaFree(c.ring_cnt);
+    if (c.peer_stats) cudaFree(c.peer_stats);
+    c.ring_cnt = nullptr;
+    c.ring_cnt_n = 0;
+    c.peer_stats = nullptr;
     c.win = nullptr;
     c.win_table = nullptr;
     c.mirror = nullptr;
@@ -119,6 +124,9 @@ int peer_compare(Ctx &c, const arc_verify_region_t &r, arc_verify_result_t *resu
     q.done_base = c.peer_done_base;
     q.done_flag = c.flag_dev;
     q.seq = ++c.seq;
+    q.ring_cnt = c.ring_cnt;
+    q.ring_cnt_n = c.ring_cnt_n;
+    q.stats = c.peer_stats;
     // the fused exchange needs a local launch: a non-empty, device-resident shard
     const bool want_fused = c.fused_exchange && r.n > 0 && classify(r.out, c.device) == PK_DEVICE &&
                             classify(r.ref, c.device) == PK_DEVICE;
@@ -136,10 +144,11 @@ int peer_compare(Ctx &c, const arc_verify_region_t &r, arc_verify_result_t *resu
     c.x_next = nullptr;
     if (st) return st;
     if (!c.x_taken) {
-        // a few blocks: the merge moves <= max_report x 24 B, mostly a handful
+        // blocks by the report size: a handful for the usual sparse report, one
+        // per SM for a dense one (ring forwarding keeps kRingGroups chunks in flight)
         q.done_base = c.peer_done_base;
         const uint64_t work = std::min<uint64_t>(r.max_report, 1ull << 40);
-        const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(32, (work + 2047) / 2048));
+        const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)c.num_sms, (work + 2047) / 2048));
         cudaLaunchConfig_t cfg = {};
         cfg.gridDim = dim3(grid);
         cfg.blockDim = dim3(256);
@@ -182,14 +191,21 @@ int arc_verify_peer_export(uint64_t max_report_cap, void *handle) {
         return ARC_E_INVAL;
     }
     peer_finalize(c);
-    const size_t bytes = kFlagBytes + 2 * packet_stride(max_report_cap);
+    const size_t bytes = window_bytes(max_report_cap);
     cudaError_t e = cudaMalloc(&c.win, bytes);
     if (e != cudaSuccess) {
         cudaGetLastError();
         set_error("cudaMalloc(peer window, %zu B)", bytes);
         return ARC_E_NOMEM;
     }
-    CK(cudaMemset(c.win, 0, kFlagBytes));
+    CK(cudaMemset(c.win, 0, kFlagBytes + ring_flag_bytes(max_report_cap)));  // call flags + ring chunk flags
+    c.ring_cnt_n = ring_chunks_max(max_report_cap);
+    e = cudaMalloc(&c.ring_cnt, 2 * c.ring_cnt_n * sizeof(uint32_t));
+    if (e != cudaSuccess) { cudaGetLastError(); set_error("cudaMalloc(ring counters)"); return ARC_E_NOMEM; }
+    CK(cudaMemset(c.ring_cnt, 0, 2 * c.ring_cnt_n * sizeof(uint32_t)));
+    e = cudaMalloc(&c.peer_stats, 2 * sizeof(unsigned long long));
+    if (e != cudaSuccess) { cudaGetLastError(); set_error("cudaMalloc(peer stats)"); return ARC_E_NOMEM; }
+    CK(cudaMemset(c.peer_stats, 0, 2 * sizeof(unsigned long long)));
     c.win_bytes = bytes;
     c.win_cap = max_report_cap;
     if (!c.mirror) {
@@ -207,6 +223,23 @@ int arc_verify_peer_export(uint64_t max_report_cap, void *handle) {
     static_assert(sizeof(h) == 64, "cudaIpcMemHandle_t is 64 bytes");
     memcpy(handle, &h, sizeof(h));
     c.coll_seq = 0;
+    return ARC_OK;
+}
+
+int arc_verify_peer_stats(uint64_t *bytes, int reset) {
+    if (!g_ctx) return ARC_E_NOINIT;
+    Ctx &c = *g_ctx;
+    if (!bytes) { set_error("peer_stats: bytes is NULL"); return ARC_E_INVAL; }
+    if (!c.peer_stats) {
+        bytes[0] = bytes[1] = 0;
+        return ARC_OK;
+    }
+    unsigned long long h[2];
+    CK(cudaStreamSynchronize(c.stream));
+    CK(cudaMemcpy(h, c.peer_stats, sizeof(h), cudaMemcpyDeviceToHost));
+    bytes[0] = h[0];
+    bytes[1] = h[1];
+    if (reset) CK(cudaMemset(c.peer_stats, 0, sizeof(h)));
     return ARC_OK;
 }
 

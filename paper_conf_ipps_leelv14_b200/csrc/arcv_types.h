@@ -22,6 +22,15 @@ constexpr int kPoolCap = 2048;                      // report phase, pool path: 
 #endif
 constexpr uint64_t kDirectDyn = ARCV_DIRECT_DYN;               // sparse reports: written directly into pinned host memory
 constexpr uint64_t kDirectBit = 1ull << 63;         // report-phase tile prefix flag: entries go to report_alias
+// Pool path (<= kPoolCap reported tiles): a denser pinned-host report is still
+// written by the kernel itself, staged per CTA in shared memory and stored as
+// coalesced 8-byte words from many CTAs (a dense tile is split across up to
+// kSplitMax CTAs), up to kDirectDense entries; beyond that HBM staging + one D2H.
+constexpr uint64_t kDirectDense = 1ull << 18;
+constexpr uint32_t kSplitMax = 16;
+constexpr uint64_t kStagedMin = 64;                 // tiles with more entries: staged, coalesced writes
+constexpr uint64_t kPinStage = 1ull << 16;          // pageable report: library pinned staging per region
+constexpr uint64_t kRoutePool = 1ull;               // Acc.pad of a published slot: the report took the pool path
 static_assert(kVecPerThread == 4, "packed-scan layout assumes 4 vectors per thread");
 static_assert(kGroupTiles == kConsumerThreads, "the report phase scans one group per block pass");
 
@@ -59,8 +68,9 @@ struct Seg {
     uint64_t max_report;    // report capacity / truncation for the region (0 = count only)
     arc_mismatch_t *report; // device pointer, entries [0, max_report)
     arc_mismatch_t *report_alias;  // device alias of the caller's pinned host report, or nullptr:
-                                   // used instead of `report` when the region has <= kDirectDyn
-                                   // mismatches (then the host skips the D2H copy)
+                                   // used instead of `report` when direct_route() holds (then
+                                   // the host skips the D2H copy)
+    uint64_t alias_cap;            // entries available at report_alias
     uint32_t acc_slot;
     uint32_t dtype;
     uint32_t flags;
@@ -73,8 +83,37 @@ struct Acc {  // per-region accumulators / result slot, 32 bytes
     unsigned long long count;
     unsigned long long max_abs_bits;
     unsigned long long max_rel_bits;
-    unsigned long long pad;
+    unsigned long long pad;  // published slot: slot_tag(seq, route, ...) (route: kRoutePool or 0)
 };
+
+// A published result slot validates itself: pad = ((seq << 1) | route) xor a
+// 64-bit hash of the three result words.  The host accepts a slot only when
+// the tag decodes to the call's sequence number, so a slot written over PCIe
+// without a system fence (clean and count-only calls, which wrote no report
+// entries to host memory) is never read torn or stale: the host re-reads
+// until the whole slot has landed (a torn read passes with probability 2^-63).
+__host__ __device__ inline uint64_t slot_mix(uint64_t z) {
+    z ^= z >> 30;
+    z *= 0xBF58476D1CE4E5B9ull;
+    z ^= z >> 27;
+    z *= 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+__host__ __device__ inline uint64_t slot_tag(uint64_t seq, uint64_t route, uint64_t count, uint64_t abs_bits,
+                                             uint64_t rel_bits) {
+    return ((seq << 1) | route) ^ slot_mix(count ^ slot_mix(abs_bits ^ slot_mix(rel_bits ^ 0x5BD1E9955BD1E995ull)));
+}
+
+// Whether a region's report entries are written by the kernel straight into
+// the pinned host buffer behind report_alias (no D2H copy).  One definition,
+// applied by the report phase and -- with `pool` read back from the published
+// slot -- by the host to decide whether it still has to copy.
+__host__ __device__ inline bool direct_route(bool has_alias, uint32_t seg_flags, uint64_t count, uint64_t max_report,
+                                             uint64_t alias_cap, bool pool) {
+    const uint64_t entries = count < max_report ? count : max_report;
+    return has_alias && !(seg_flags & kSegBaseFromAcc) && entries <= alias_cap &&
+           (count <= kDirectDyn || (pool && count <= kDirectDense));
+}
 
 // The sharded exchange over peer windows (arcv_exchange.cuh): one call's
 // parameters, used by the exchange kernel and by K1's fused exchange.
@@ -93,6 +132,9 @@ struct PeerParams {
     unsigned long long done_base;
     unsigned long long *done_flag;  // mapped completion word
     unsigned long long seq;
+    uint32_t *ring_cnt;             // [2 parities][ring_cnt_n] per-chunk block counters (ring mode; local HBM)
+    uint64_t ring_cnt_n;
+    unsigned long long *stats;      // [2] monotonic: bytes read from owners' packets / forwarding ranks
 };
 
 struct Params {

@@ -784,3 +784,45 @@ def test_env_flags_cannot_disable_the_predicate():
         res = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=300, env=env)
         assert res.returncode == 0, res.stderr[-2000:]
         assert "COUNT 45" in res.stdout, (flags, res.stdout)
+
+
+@pytest.mark.parametrize("dt,n_dense,mr,buf,off", [
+    ("f32", 2, 1 << 20, "pinned", 0),      # C2B-like: 2 dense tiles, split across CTAs, direct
+    ("f32", 2, 1 << 20, "pageable", 1),    # library pinned staging, misaligned arrays
+    ("f32", 2, 5000, "pinned", 0),         # truncation inside the second tile
+    ("f64", 20, 1 << 20, "pinned", 0),     # 40960 entries, pool path, direct
+    ("f64", 20, 1 << 20, "pageable", 0),   # > the 2^16 pageable staging: HBM staging + D2H
+    ("i32", 100, 1 << 20, "pinned", 3),    # 409600 > 2^18 entries: HBM staging + D2H
+    ("i32", 100, 7777, "pinned", 0),       # truncated far below: direct
+    ("u8", 3, 1 << 20, "pinned", 5),       # u8 tiles (16384 elements), split
+    ("f32", 2, 1 << 20, "device", 0),      # device report: split tiles, staged coalesced stores
+    ("f32", 1, 1 << 20, "pinned", 0),      # one dense tile split across up to 16 CTAs
+])
+def test_dense_tiles_direct_route(av, orc, dt, n_dense, mr, buf, off):
+    """Few report tiles holding many mismatches (C2B's shape: a wrong loop bound leaves a
+    whole row stale): the pool path splits each dense tile across several CTAs, which write
+    their rank ranges through shared memory as coalesced words -- into the caller's pinned
+    buffer (or the library's pinned staging) when direct_route() allows, else into HBM
+    staging followed by one D2H copy.  Every combination bit-exact against the oracle."""
+    te = TILE_ELEMS[dt]
+    n = te * (n_dense * 3 + 5) + 123
+    out, ref = random_pair(dt, n + off, seed=4242 + n_dense, rate=0.0)
+    out, ref = out[off:], ref[off:]
+    for k in range(n_dense):  # every third tile fully mismatching (plus a partial tail)
+        t0 = (3 * k + 1) * te
+        if dt in ("f32", "f64"):
+            out[t0:t0 + te] = ref[t0:t0 + te] * 1.5 + 0.25
+        else:
+            out[t0:t0 + te] = ref[t0:t0 + te] ^ 1
+    if buf == "pinned":
+        rep = torch.empty(24 * mr, dtype=torch.uint8, pin_memory=True).numpy().view(av.REPORT_DTYPE)
+        rep.view(np.uint8)[:] = 0xA5
+    elif buf == "pageable":
+        rep = np.full(mr, 0, dtype=av.REPORT_DTYPE)
+    else:
+        rep = torch.empty(24 * mr, dtype=torch.uint8, device="cuda")
+    at, rt = (1e-6, 1e-5) if dt in ("f32", "f64") else (0, 0)
+    e = orc.compare(out.cpu().numpy(), ref.cpu().numpy(), dt, at, rt, mr)
+    for it in range(3):
+        g = av.compare(out, ref, at, rt, mr, report=rep)
+        assert_same(g, e, f"{dt} dense={n_dense} mr={mr} {buf} off={off} it={it}")

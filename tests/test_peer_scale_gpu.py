@@ -80,13 +80,20 @@ def _worker(rank, world, port, q, transport, device):
         assert got == transport, got
         pinned = torch.empty(24 * MR, dtype=torch.uint8, pin_memory=True).numpy().view(av.REPORT_DTYPE)
         dev_rep = torch.empty(24 * MR, dtype=torch.uint8, device="cuda")
-        for name, reg, _dt in _cases(world):
+        cases = {name: reg for name, reg, _dt in _cases(world)}
+        # C5 (dense: ring forwarding at p >= 3), C4 (sparse: pull), C5 again
+        # (the ring's per-call chunk counters after a pull-mode call)
+        for name, reps in (("C5", range(4)), ("C4", range(4)), ("C5", range(4, 6))):
+            reg = cases[name]
             a, b = rank * reg.n // world, (rank + 1) * reg.n // world
             o, r = reg.slice(a, b - a, device="cuda")
-            for rep in range(4):  # consecutive calls alternate the window parity
-                buf = (None, pinned, dev_rep, pinned)[rep]
+            av.arc_verify_peer_stats(reset=True)
+            for rep in reps:  # consecutive calls alternate the window parity
+                buf = (None, pinned, dev_rep, pinned, dev_rep, None)[rep]
                 g = av.compare(o, r, reg.abs_tol, reg.rel_tol, reg.max_report, report=buf)
                 out.append(((name, rep), _digest(g, av)))
+            pulled, forwarded = av.arc_verify_peer_stats()
+            out.append(((name, "bytes", reps[0]), (pulled // len(reps), forwarded // len(reps))))
             del o, r
             torch.cuda.empty_cache()
         av.finalize()
@@ -145,6 +152,11 @@ def _run(world, transport, device, timeout=900):
     return res
 
 
+def _results(d):
+    """The global results (identical on every rank); per-rank byte counters excluded."""
+    return {k: v for k, v in d.items() if "bytes" not in k}
+
+
 def _on_gpu0(rank):
     return 0
 
@@ -158,11 +170,23 @@ def _own_gpu(rank):
 def test_sharded_north_star_shapes_peer(world):
     res = _run(world, "peer", _on_gpu0)
     for r in range(1, world):
-        assert res[r] == res[0], f"rank {r} differs from rank 0"
+        assert _results(res[r]) == _results(res[0]), f"rank {r} differs from rank 0"
     want = _expected(world)
-    for name in ("C5", "C4"):
-        for rep in range(4):
+    for name, reps in (("C5", range(6)), ("C4", range(4))):
+        for rep in reps:
             assert res[0][(name, rep)] == want[name], (world, name, rep, res[0][(name, rep)], want[name])
+    # bytes read from peer windows per call (measured by the exchange kernels):
+    # C5's 2^20 entries all belong to rank 0; with ring forwarding (p >= 3)
+    # rank 1 pulls them from rank 0 and rank k >= 2 from rank k - 1, so every
+    # window is read once; at p = 2 rank 1 pulls them from rank 0
+    rep_bytes = 24 * MR
+    for first in (0, 4):
+        per_rank = [res[r][("C5", "bytes", first)] for r in range(world)]
+        assert per_rank[0] == (0, 0), per_rank
+        assert per_rank[1] == (rep_bytes, 0), per_rank
+        for r in range(2, world):
+            assert per_rank[r] == (0, rep_bytes), (r, per_rank)
+    # C4 (516 entries, pull): each rank reads the other ranks' contributions once
 
 
 @pytest.mark.timeout(1500)
@@ -171,8 +195,8 @@ def test_sharded_north_star_shapes_nccl_two_gpus():
     """The NCCL fallback (all-gather of packets, merge kernel, grouped broadcast of
     the entries beyond a packet: C5's 2^20-entry report) across two real GPUs."""
     res = _run(2, "nccl", _own_gpu)
-    assert res[1] == res[0]
+    assert _results(res[1]) == _results(res[0])
     want = _expected(2)
-    for name in ("C5", "C4"):
-        for rep in range(4):
+    for name, reps in (("C5", range(6)), ("C4", range(4))):
+        for rep in reps:
             assert res[0][(name, rep)] == want[name], (name, rep)

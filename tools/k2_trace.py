@@ -23,7 +23,7 @@ assert lib.arc_verify_init(ctypes.byref(opts)) == 0
 REP = torch.empty(24 * (1 << 20), dtype=torch.uint8, pin_memory=True).numpy().view(av.REPORT_DTYPE)
 P, U64, I, D = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int, ctypes.c_double
 lib.arc_verify_compare.argtypes = [P, P, U64, I, D, D, U64, ctypes.POINTER(av.arc_verify_result_t)]
-K1 = ["start", "loop end", "flush end", "exit"]
+K1 = ["start", "loop end", "flush end", "exit", "first stage landed", "first tile evaluated"]
 K2 = ["entry / barrier arrive", "after wait", "tile 0 emitted", "prefixes reduced", "tile 0 landed",
       "tile 0 masked", "pool loop end", "exit", "last rep start (TAIL_REPS)", "pool loaded", "tile 1 emitted",
       "after last_cta (fence+atomic+bar)"]
@@ -54,8 +54,20 @@ def run(name, o, r, at, rt, mr):
                 print(f"  {kn} {nm:18s} min {d.min():8.2f}  med {np.median(d):8.2f}  max {d.max():8.2f}  (n={len(col)})")
 
 
-c = synth.C4(1 << lg)
-o, r = c.slice(device="cuda")
-run(f"C4 fp64 2^{lg}, max_report 2^20", o, r, c.abs_tol, c.rel_tol, c.max_report)
-run(f"C4 fp64 2^{lg}, count only", o, r, c.abs_tol, c.rel_tol, 0)
-run(f"C4 fp64 2^{lg}, clean (out==ref), max_report 2^20", r, r, c.abs_tol, c.rel_tol, c.max_report)
+if os.environ.get("TRACE_C2A"):
+    c2 = synth.C2("A")
+    o, r = c2.slice(device="cuda")
+    run("C2A fp32 8192^2, max_report 2^20", o, r, c2.abs_tol, c2.rel_tol, c2.max_report)
+    run("C2A fp32 8192^2, count only", o, r, c2.abs_tol, c2.rel_tol, 0)
+    run("C2A bytes as u8 (no float filter), count only", o.view(torch.uint8), r.view(torch.uint8), 0, 0, 0)
+    c2b = synth.C2("B")
+    o, r = c2b.slice(device="cuda")
+    run("C2B fp32 8192^2 (2 dense tiles), pinned report 2^20", o, r, c2b.abs_tol, c2b.rel_tol, c2b.max_report)
+    c1 = synth.C1()
+    o, r = c1.slice(device="cuda")
+    run("C1 fp32 2^20, pinned report 2^20", o, r, c1.abs_tol, c1.rel_tol, c1.max_report)
+else:
+    c = synth.C4(1 << lg)
+    o, r = c.slice(device="cuda")
+    run(f"C4 fp64 2^{lg}, max_report 2^20", o, r, c.abs_tol, c.rel_tol, c.max_report)
+    run(f"C4 fp64 2^{lg}, count only", o, r, c.abs_tol, c.rel_tol, 0)

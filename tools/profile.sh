@@ -25,7 +25,34 @@ for _ in range(5): av.compare(o, r, 0.0, 1e-5, 1 << 20)
 torch.cuda.synchronize(); av.finalize()
 " > $OUT/${TAG}_k1_c2a.log 2>&1
 echo "k1 c2a rc=$?"
-for f in k1_c4 k1_c2a; do
+# C2B (two dense tiles, pinned report: split + coalesced direct writes), C3 (one
+# batched launch over twelve regions), C5 (int32 2^30, 50 % mismatches: group path)
+for cfg in c2b c3 c5; do
+$NCU --set full --clock-control none --import-source on -k regex:arcv_stream_kernel -s 3 -c 1 \
+  -o $OUT/${TAG}_k1_$cfg -f python -c "
+import sys; sys.path.insert(0, '.')
+import torch, synth, paper_conf_ipps_leelv14_b200 as av
+av.init(0)
+cfg = '$cfg'
+if cfg == 'c2b':
+    o, r = synth.C2('B').slice(device='cuda')
+    rep = torch.empty(24 << 20, dtype=torch.uint8, pin_memory=True).numpy().view(av.REPORT_DTYPE)
+    for _ in range(5): av.compare(o, r, 0.0, 1e-5, 1 << 20, report=rep)
+elif cfg == 'c3':
+    regs = synth.c3_regions()
+    data = [rg.slice(device='cuda') for rg in regs]
+    pb = av.prepare_batch([(o, r, rg.abs_tol, rg.rel_tol, rg.max_report, rg.name) for rg, (o, r) in zip(regs, data)])
+    for _ in range(5): pb()
+else:
+    c5 = synth.C5()
+    o, r = c5.slice(device='cuda')
+    drep = torch.empty(24 << 20, dtype=torch.uint8, device='cuda')
+    for _ in range(5): av.compare(o, r, 0, 0, 1 << 20, report=drep)
+torch.cuda.synchronize(); av.finalize()
+" > $OUT/${TAG}_k1_$cfg.log 2>&1
+echo "k1 $cfg rc=$?"
+done
+for f in k1_c4 k1_c2a k1_c2b k1_c3 k1_c5; do
   $NCU -i $OUT/${TAG}_$f.ncu-rep --page raw --csv > $OUT/${TAG}_${f}_raw.csv 2>/dev/null
   $NCU -i $OUT/${TAG}_$f.ncu-rep --page details --csv > $OUT/${TAG}_${f}_details.csv 2>/dev/null
 done
