@@ -757,6 +757,14 @@ __device__ __noinline__ void compact_tile(const Seg &g, const StageInfo &si, con
 // matches), so the in-tile ranks agree with K1's counts.
 // Scalars by value: references to SegHot / StageInfo would put them in local
 // memory (the function is not inlined) and reload them every iteration.
+// -DARCV_MASK_UNROLL=N: unroll the mask loops N-fold (A/B builds; default 1:
+// compact code, cold once per CTA).
+#ifndef ARCV_MASK_UNROLL
+#define ARCV_MASK_UNROLL 1
+#endif
+#define ARCV_PRAGMA_(x) _Pragma(#x)
+#define ARCV_UNROLL_(n) ARCV_PRAGMA_(unroll n)
+#define ARCV_UNROLL(n) ARCV_UNROLL_(n)
 template <typename T>
 __device__ __noinline__ uint64_t mask_tile(const uint8_t *so, const uint8_t *sr, uint32_t count, uint32_t off_o,
                                            uint32_t off_r, int tid, double abs_tol, double rel_tol, uint32_t cflags,
@@ -776,7 +784,7 @@ __device__ __noinline__ uint64_t mask_tile(const uint8_t *so, const uint8_t *sr,
             return mask;
         }
     }
-#pragma unroll 1
+    ARCV_UNROLL(ARCV_MASK_UNROLL)
     for (int b = 0; b < kVecPerThread * EPV; ++b) {
         const uint32_t e = (uint32_t)(((b / EPV) * kConsumerThreads + tid) * EPV + (b % EPV));
         if (e >= count) continue;
@@ -881,7 +889,7 @@ __device__ __noinline__ uint64_t mask_tile_half(const uint8_t *so, const uint8_t
                                                 uint32_t cflags, double minv, double lo, double hi) {
     constexpr int EPV = 16 / sizeof(T);
     uint64_t mask = 0;
-#pragma unroll 1
+    ARCV_UNROLL(ARCV_MASK_UNROLL)
     for (int b = 0; b < 2 * kVecPerThread * EPV; ++b) {
         const uint32_t e = (uint32_t)(((b / EPV) * (kConsumerThreads / 2) + gt) * EPV + (b % EPV));
         if (e >= count) continue;
@@ -1074,6 +1082,12 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
     };
 
     const uint32_t n_nz = *(volatile uint32_t *)p.nz_cnt;
+    // the reporting regions' final counts (the pool path's split decision),
+    // loaded alongside n_nz: no extra round trip on the critical path
+    uint64_t tot_cnt = 0;
+    if (p.n_segs <= (uint32_t)kMaxInlineSegs)
+        for (uint32_t sgi = 0; sgi < p.n_segs; ++sgi)
+            if (segs[sgi].max_report) tot_cnt += __ldcg(&p.acc[segs[sgi].acc_slot].count);
     const uint32_t G = gridDim.x, b = blockIdx.x;
     if (n_nz <= (uint32_t)kPoolCap) {
         // ------------------------------------------------------ pool path
@@ -1084,12 +1098,9 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
         // written by S SMs; work item i = pool entry i / S, part i % S.  Every
         // CTA derives the same S from the final counts.
         uint32_t S = 1u;
-        if (n_nz > 0 && 2 * n_nz <= G && p.n_segs <= (uint32_t)kMaxInlineSegs) {
-            uint64_t tot_cnt = 0;
-            for (uint32_t sgi = 0; sgi < p.n_segs; ++sgi)
-                if (segs[sgi].max_report) tot_cnt += __ldcg(&p.acc[segs[sgi].acc_slot].count);
-            if (tot_cnt > (uint64_t)n_nz * kStagedMin) S = min(kSplitMax, G / n_nz);
-        }
+        if (n_nz > 0 && 2 * n_nz <= G && p.n_segs <= (uint32_t)kMaxInlineSegs &&
+            tot_cnt > (uint64_t)n_nz * kStagedMin)
+            S = min(kSplitMax, G / n_nz);
         const uint32_t n_items = n_nz * S;
 #if defined(ARCV_TAIL_REPS)
       // diagnostic: run the (idempotent) pool path again, stamps from the last run

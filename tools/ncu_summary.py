@@ -43,9 +43,11 @@ def main():
         k = out[name]
         try:  # derived: DRAM bytes / L2 read sectors vs 32-byte sectors of DRAM reads
             num = lambda s: float(s.split()[0].replace(",", ""))
-            if "dram__sectors_read.sum" in k and "lts__t_sectors_op_read.sum" in k:
-                k["derived_l2_read_sectors_per_dram_read_sector"] = round(
-                    num(k["lts__t_sectors_op_read.sum"]) / max(num(k["dram__sectors_read.sum"]), 1), 4)
+            if "dram__sectors_read.sum" in k and "lts__t_sectors_srcunit_tex_op_read.sum" in k:
+                # ~1.0: every 32-byte sector the SMs read through L2 came from DRAM exactly once
+                k["derived_l2_tex_read_sectors_per_dram_read_sector"] = round(
+                    num(k["lts__t_sectors_srcunit_tex_op_read.sum"]) / max(num(k["dram__sectors_read.sum"]), 1), 5)
+                k["derived_dram_read_bytes_from_sectors"] = int(32 * num(k["dram__sectors_read.sum"]))
             if "lts__t_sectors_op_read.sum" in k and "lts__t_requests_op_read.sum" in k:
                 k["derived_l2_sectors_per_request"] = round(
                     num(k["lts__t_sectors_op_read.sum"]) / max(num(k["lts__t_requests_op_read.sum"]), 1), 3)

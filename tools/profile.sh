@@ -55,5 +55,7 @@ done
 for f in k1_c4 k1_c2a k1_c2b k1_c3 k1_c5; do
   $NCU -i $OUT/${TAG}_$f.ncu-rep --page raw --csv > $OUT/${TAG}_${f}_raw.csv 2>/dev/null
   $NCU -i $OUT/${TAG}_$f.ncu-rep --page details --csv > $OUT/${TAG}_${f}_details.csv 2>/dev/null
+  # the .ncu-rep files are large (gpurun copies back <= 64 MiB): keep them only on request
+  [ -n "${KEEP_REP:-}" ] || rm -f $OUT/${TAG}_$f.ncu-rep
 done
 echo done
