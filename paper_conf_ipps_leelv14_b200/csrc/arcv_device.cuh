@@ -110,8 +110,10 @@ __device__ __forceinline__ void fence_sys() {
 // Diagnostic phase trace (A/B builds only, -DARCV_TRACE=1): %globaltimer stamps
 // per CTA, read by arc_verify_debug_trace.  Compiled out otherwise.
 #if defined(ARCV_TRACE) && ARCV_TRACE
-constexpr int kTraceCtas = 1024, kTracePts = 12;
-__device__ unsigned long long g_trace[2][kTraceCtas][kTracePts];  // [kernel][cta][point]
+constexpr int kTraceCtas = 1024, kTracePts = 32, kTraceRows = 3;
+// [row][cta][point]: row 0 K1, row 1 report phase, row 2 region switches
+// (point 2 seg: switched into segment seg, 2 seg + 1: its first tile evaluated; seg < 16)
+__device__ unsigned long long g_trace[kTraceRows][kTraceCtas][kTracePts];
 #define ARCV_STAMP(k, pt)                                                                      \
     do {                                                                                       \
         unsigned long long t_;                                                                 \
@@ -684,7 +686,7 @@ __device__ __forceinline__ uint64_t block_excl_scan(uint64_t v, uint64_t *s_w, u
 // scatter).  Called by all 256 consumer threads (it synchronises them).
 constexpr int kOutEntries = 1024;
 template <typename T>
-__device__ __noinline__ void compact_tile(const Seg &g, const StageInfo &si, const uint8_t *so, const uint8_t *sr,
+__device__ __noinline__ void compact_tile(const Seg &g, uint64_t si_elem_begin, uint32_t si_off_o, uint32_t si_off_r, const uint8_t *so, const uint8_t *sr,
                                           uint64_t mask, uint64_t excl, uint64_t *s_w, int tid, uint64_t rlo,
                                           uint64_t rhi, arc_mismatch_t *obuf) {
     constexpr int EPV = 16 / sizeof(T);
@@ -713,9 +715,9 @@ __device__ __noinline__ void compact_tile(const Seg &g, const StageInfo &si, con
                 if (rank >= r0 && rank < r1) {
                     const uint32_t te = (uint32_t)((k * kConsumerThreads + tid) * EPV + j);
                     arc_mismatch_t e;
-                    e.index = g.index_base + si.elem_begin + te;
-                    e.out_bits = raw_bits<T>(*reinterpret_cast<const T *>(so + si.off_o + te * sizeof(T)));
-                    e.ref_bits = raw_bits<T>(*reinterpret_cast<const T *>(sr + si.off_r + te * sizeof(T)));
+                    e.index = g.index_base + si_elem_begin + te;
+                    e.out_bits = raw_bits<T>(*reinterpret_cast<const T *>(so + si_off_o + te * sizeof(T)));
+                    e.ref_bits = raw_bits<T>(*reinterpret_cast<const T *>(sr + si_off_r + te * sizeof(T)));
                     obuf[rank - r0] = e;
                 }
             }
@@ -739,10 +741,10 @@ __device__ __noinline__ void compact_tile(const Seg &g, const StageInfo &si, con
         const uint64_t gi = excl + rank;
         if (gi < g.max_report) {
             const uint32_t te = (uint32_t)((k * kConsumerThreads + tid) * EPV + j);  // tile element
-            const T xo = *reinterpret_cast<const T *>(so + si.off_o + te * sizeof(T));  // from the stage
-            const T xr = *reinterpret_cast<const T *>(sr + si.off_r + te * sizeof(T));
+            const T xo = *reinterpret_cast<const T *>(so + si_off_o + te * sizeof(T));  // from the stage
+            const T xr = *reinterpret_cast<const T *>(sr + si_off_r + te * sizeof(T));
             arc_mismatch_t *dst = rep + gi;
-            dst->index = g.index_base + si.elem_begin + te;
+            dst->index = g.index_base + si_elem_begin + te;
             dst->out_bits = raw_bits<T>(xo);
             dst->ref_bits = raw_bits<T>(xr);
         }
@@ -912,7 +914,7 @@ __device__ __noinline__ uint64_t mask_tile_half(const uint8_t *so, const uint8_t
 }
 
 template <typename T>
-__device__ __noinline__ void compact_tile_half(const Seg &g, const StageInfo &si, const uint8_t *so,
+__device__ __noinline__ void compact_tile_half(const Seg &g, uint64_t si_elem_begin, uint32_t si_off_o, uint32_t si_off_r, const uint8_t *so,
                                                const uint8_t *sr, uint64_t mask, uint64_t excl, uint64_t *s_w,
                                                int gt, int grp) {
     constexpr int EPV = 16 / sizeof(T);
@@ -941,10 +943,10 @@ __device__ __noinline__ void compact_tile_half(const Seg &g, const StageInfo &si
         const uint64_t gi = excl + rank;
         if (gi < g.max_report) {
             const uint32_t te = (uint32_t)((k * (kConsumerThreads / 2) + gt) * EPV + j);
-            const T xo = *reinterpret_cast<const T *>(so + si.off_o + te * sizeof(T));
-            const T xr = *reinterpret_cast<const T *>(sr + si.off_r + te * sizeof(T));
+            const T xo = *reinterpret_cast<const T *>(so + si_off_o + te * sizeof(T));
+            const T xr = *reinterpret_cast<const T *>(sr + si_off_r + te * sizeof(T));
             arc_mismatch_t *dst = rep + gi;
-            dst->index = g.index_base + si.elem_begin + te;
+            dst->index = g.index_base + si_elem_begin + te;
             dst->out_bits = raw_bits<T>(xo);
             dst->ref_bits = raw_bits<T>(xr);
         }
@@ -957,7 +959,7 @@ __device__ __forceinline__ void emit_half_any(const Seg &g, const StageInfo &si,
     {                                                                                                         \
         const uint64_t mk = mask_tile_half<T>(so, so + kStageArrayBytes, si.count, si.off_o, si.off_r, gt,     \
                                               g.abs_tol, g.rel_tol, g.cflags, g.minv, g.lo, g.hi);            \
-        compact_tile_half<T>(g, si, so, so + kStageArrayBytes, mk, excl, s_w, gt, grp);                      \
+        compact_tile_half<T>(g, si.elem_begin, si.off_o, si.off_r, so, so + kStageArrayBytes, mk, excl, s_w, gt, grp);                      \
     }
     switch (g.dtype) {
         case ARC_F32: ARCV_HALF(float) break;
@@ -972,11 +974,11 @@ __device__ __forceinline__ void compact_any(const Seg &g, const StageInfo &si, c
                                             uint64_t mask, uint64_t excl, uint64_t *s_w, int tid, uint64_t rlo,
                                             uint64_t rhi, arc_mismatch_t *obuf) {
     switch (g.dtype) {
-        case ARC_F32: compact_tile<float>(g, si, so, sr, mask, excl, s_w, tid, rlo, rhi, obuf); break;
-        case ARC_F64: compact_tile<double>(g, si, so, sr, mask, excl, s_w, tid, rlo, rhi, obuf); break;
-        case ARC_I32: compact_tile<int32_t>(g, si, so, sr, mask, excl, s_w, tid, rlo, rhi, obuf); break;
-        case ARC_I64: compact_tile<int64_t>(g, si, so, sr, mask, excl, s_w, tid, rlo, rhi, obuf); break;
-        default: compact_tile<uint8_t>(g, si, so, sr, mask, excl, s_w, tid, rlo, rhi, obuf); break;
+        case ARC_F32: compact_tile<float>(g, si.elem_begin, si.off_o, si.off_r, so, sr, mask, excl, s_w, tid, rlo, rhi, obuf); break;
+        case ARC_F64: compact_tile<double>(g, si.elem_begin, si.off_o, si.off_r, so, sr, mask, excl, s_w, tid, rlo, rhi, obuf); break;
+        case ARC_I32: compact_tile<int32_t>(g, si.elem_begin, si.off_o, si.off_r, so, sr, mask, excl, s_w, tid, rlo, rhi, obuf); break;
+        case ARC_I64: compact_tile<int64_t>(g, si.elem_begin, si.off_o, si.off_r, so, sr, mask, excl, s_w, tid, rlo, rhi, obuf); break;
+        default: compact_tile<uint8_t>(g, si.elem_begin, si.off_o, si.off_r, so, sr, mask, excl, s_w, tid, rlo, rhi, obuf); break;
     }
 }
 
@@ -1110,23 +1112,28 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
 #endif
         const uint32_t n_own = n_items > b ? (n_items - b + G - 1) / G : 0u;
         auto entry_of = [&](uint32_t j) { return (b + j * G) / S; };  // my j-th item's pool entry
-        if (tid == 0 && n_own > 0) {  // both key loads in flight before the first issue
-            const uint64_t k0 = __ldcg(p.nz_list + 2 * entry_of(0));
-            const uint64_t k1 = n_own > 1 ? __ldcg(p.nz_list + 2 * entry_of(1)) : 0ull;
-            issue(k0, 0);
-            if (n_own > 1) issue(k1, 1);
-        }
-        // the whole pool in registers, all loads in flight at once: entry
-        // tid + u * 256 = {seg << 40 | tile, count}; absent entries never match
+        const ulonglong2 *nzl = reinterpret_cast<const ulonglong2 *>(p.nz_list);
+        // One round trip for everything the prefixes and the first re-reads
+        // need: the CTA's first two pool entries (every thread: they are also
+        // the keys of the prefix pass) and the whole pool in registers (entry
+        // tid + u * 256 = {seg << 40 | tile, count}; absent entries never
+        // match), all loads in flight before thread 0 issues the re-reads.
+        ulonglong2 kv[2] = {make_ulonglong2(~0ull - 1, 0ull), make_ulonglong2(~0ull - 1, 0ull)};
+        if (n_own > 0) kv[0] = __ldcg(nzl + entry_of(0));
+        if (n_own > 1) kv[1] = __ldcg(nzl + entry_of(1));
         constexpr int kPer = kPoolCap / kConsumerThreads;
         uint64_t pk[kPer], pc[kPer];
 #pragma unroll
         for (int u = 0; u < kPer; ++u) {
             const uint32_t i = (uint32_t)tid + (uint32_t)u * kConsumerThreads;
             ulonglong2 e = make_ulonglong2(~0ull, 0ull);
-            if (i < n_nz) e = __ldcg(reinterpret_cast<const ulonglong2 *>(p.nz_list) + i);
+            if (i < n_nz) e = __ldcg(nzl + i);
             pk[u] = e.x;
             pc[u] = e.y;
+        }
+        if (tid == 0) {
+            if (n_own > 0) issue(kv[0].x, 0);
+            if (n_own > 1) issue(kv[1].x, 1);
         }
 #if defined(ARCV_TRACE) && ARCV_TRACE
         if (tid == 0 && pk[0] != 1ull) ARCV_STAMP(1, 9);  // waits for the first pool load
@@ -1138,10 +1145,9 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
 #pragma unroll
             for (int q = 0; q < 2; ++q) {
                 if ((uint32_t)q < m) {
-                    const uint32_t e = entry_of(j0 + q);
-                    const ulonglong2 kv = __ldcg(reinterpret_cast<const ulonglong2 *>(p.nz_list) + e);
-                    key[q] = kv.x;
-                    tcn[q] = kv.y;
+                    const ulonglong2 e = j0 == 0 ? kv[q] : __ldcg(nzl + entry_of(j0 + q));
+                    key[q] = e.x;
+                    tcn[q] = e.y;
                     part[q] = (b + (j0 + q) * G) % S;
                 } else {
                     key[q] = ~0ull - 1;
@@ -1451,6 +1457,10 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
         const StageInfo si = info[s];
         if (si.tile == ~0ull) break;
         if ((int)si.seg != cur) {
+#if defined(ARCV_TRACE) && ARCV_TRACE
+            if (ctid == 0 && si.seg < 16 && g_trace[2][blockIdx.x < (unsigned)kTraceCtas ? blockIdx.x : 0][2 * si.seg] == 0)
+                ARCV_STAMP(2, 2 * si.seg);
+#endif
             const uint32_t slot = segs[si.seg].acc_slot;
             if (cur >= 0 && slot != g.acc_slot) flush_acc(p.acc, g.acc_slot, g.dtype, acc, ctid, s_red_u, s_red_d);
             cur = (int)si.seg;
@@ -1461,6 +1471,10 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
         const uint32_t cnt = (p.flags & kFlagProbe) ? 0u : eval_any(so, so + kStageArrayBytes, si, ctid, g, acc);
         acc.count += cnt;
         if (ctid == 0 && i == 0) ARCV_STAMP(0, 5);
+#if defined(ARCV_TRACE) && ARCV_TRACE
+        if (ctid == 0 && si.seg < 16 && g_trace[2][blockIdx.x < (unsigned)kTraceCtas ? blockIdx.x : 0][2 * si.seg + 1] == 0)
+            ARCV_STAMP(2, 2 * si.seg + 1);
+#endif
         if (g.max_report != 0) {
             // Per-tile count for the report phase: warps fold their counts into the stage's
             // shared word (arrivals << 24 | count); the last warp publishes the

@@ -32,13 +32,13 @@ K2 = ["entry / barrier arrive", "after wait", "tile 0 emitted", "prefixes reduce
 def run(name, o, r, at, rt, mr):
     res = av.arc_verify_result_t()
     res.report = REP.ctypes.data
-    buf = np.zeros((2, 1024, 12), dtype=np.uint64)
+    buf = np.zeros((3, 1024, 32), dtype=np.uint64)
     for it in range(5):
         if it == 4:  # clear the stamps: the traced call is the last one
             lib.arc_verify_debug_trace(buf.ctypes.data_as(ctypes.POINTER(ctypes.c_ulonglong)))
         assert lib.arc_verify_compare(o.data_ptr(), r.data_ptr(), o.numel(), av.dtype_code(o), at, rt, mr,
                                       ctypes.byref(res)) == 0
-    buf = np.zeros((2, 1024, 12), dtype=np.uint64)
+    buf = np.zeros((3, 1024, 32), dtype=np.uint64)
     assert lib.arc_verify_debug_trace(buf.ctypes.data_as(ctypes.POINTER(ctypes.c_ulonglong))) == 0
     t = buf.astype(np.float64)
     k1 = t[0][t[0][:, 0] > 0]
