@@ -1449,7 +1449,6 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
     int cur = -1;
     SegHot g;
     if (ctid == 0) ARCV_STAMP(0, 0);
-
     for (uint32_t i = 0;; ++i) {
         const int s = i % S;
         mbar_wait(&full_bar[s], (i / S) & 1);
