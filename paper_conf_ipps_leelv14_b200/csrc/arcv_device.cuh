@@ -135,6 +135,20 @@ __device__ __forceinline__ double warp_max_f64(double v) {
     return v;
 }
 
+#define ARCV_PRAGMA_(x) _Pragma(#x)
+#define ARCV_UNROLL_(n) ARCV_PRAGMA_(unroll n)
+#define ARCV_UNROLL(n) ARCV_UNROLL_(n)
+// Code-size knobs (A/B builds): unroll factors of the per-tile vector loop
+// (default: all kVecPerThread = 4 vectors) and of the seeding scan (default:
+// all elements).  Smaller code = fewer cold instruction lines on the first
+// tile of a region (profiles/r02i_stall_summary.txt).
+#ifndef ARCV_EVAL_UNROLL
+#define ARCV_EVAL_UNROLL 4
+#endif
+#ifndef ARCV_SEED_UNROLL
+#define ARCV_SEED_UNROLL 64
+#endif
+
 // ------------------------------------------------------------ element predicate
 struct ThreadAcc {
     uint64_t count;
@@ -296,6 +310,7 @@ __device__ __forceinline__ void seed_bounds(const uint8_t *so, const uint8_t *sr
     acc.seeded = true;
     float best_d = -1.f, best_r = -1.f;
     int bd = -1, br = -1;
+    ARCV_UNROLL(ARCV_SEED_UNROLL)
     for (int b = 0; b < kVecPerThread * EPV; ++b) {
         const uint32_t e = (uint32_t)(((b / EPV) * kConsumerThreads + ctid) * EPV + (b % EPV));
         if (e >= cnt) continue;
@@ -364,7 +379,7 @@ __device__ __forceinline__ uint32_t eval_tile(const uint8_t *so, const uint8_t *
             rel_form = g.rel_tol > 0.0;
         }
     }
-#pragma unroll
+    ARCV_UNROLL(ARCV_EVAL_UNROLL)
     for (int k = 0; k < kVecPerThread; ++k) {
         const uint32_t v = k * kConsumerThreads + ctid;
         T xo[EPV], xr[EPV];
@@ -764,9 +779,6 @@ __device__ __noinline__ void compact_tile(const Seg &g, uint64_t si_elem_begin, 
 #ifndef ARCV_MASK_UNROLL
 #define ARCV_MASK_UNROLL 1
 #endif
-#define ARCV_PRAGMA_(x) _Pragma(#x)
-#define ARCV_UNROLL_(n) ARCV_PRAGMA_(unroll n)
-#define ARCV_UNROLL(n) ARCV_UNROLL_(n)
 template <typename T>
 __device__ __noinline__ uint64_t mask_tile(const uint8_t *so, const uint8_t *sr, uint32_t count, uint32_t off_o,
                                            uint32_t off_r, int tid, double abs_tol, double rel_tol, uint32_t cflags,

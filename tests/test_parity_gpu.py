@@ -826,3 +826,37 @@ def test_dense_tiles_direct_route(av, orc, dt, n_dense, mr, buf, off):
     for it in range(3):
         g = av.compare(out, ref, at, rt, mr, report=rep)
         assert_same(g, e, f"{dt} dense={n_dense} mr={mr} {buf} off={off} it={it}")
+
+
+@pytest.mark.parametrize("kind", ["checks", "batch"])
+def test_dense_tiles_checks_and_batches(av, orc, kind):
+    """The split / staged dense-tile route combined with the N2 checks (minValueToCheck and
+    value bounds remove some mismatches inside the dense tiles, so K1's counts and the
+    report phase's ranks must agree under the checks) and inside a batch (a dense region
+    and a sparse one sharing the pool, each with its own pinned report)."""
+    te = TILE_ELEMS["f32"]
+    n = te * 9 + 77
+    out, ref = random_pair("f32", n, seed=777, rate=0.0)
+    for t in (2, 6):
+        out[t * te:(t + 1) * te] = ref[t * te:(t + 1) * te] * 1.5 + 0.25
+    mr = 1 << 20
+    pin = lambda cap: torch.empty(24 * cap, dtype=torch.uint8, pin_memory=True).numpy().view(av.REPORT_DTYPE)
+    if kind == "checks":
+        rep = pin(mr)
+        for mv, bounds in ((0.5, None), (None, (-0.2, 0.9)), (0.25, (0.0, 1.0))):
+            e = orc.compare(out.cpu().numpy(), ref.cpu().numpy(), "f32", 1e-6, 1e-5, mr, min_value=mv, bounds=bounds)
+            g = av.compare(out, ref, 1e-6, 1e-5, mr, report=rep, min_value=mv, bounds=bounds)
+            assert_same(g, e, f"dense + checks {mv} {bounds}")
+    else:
+        o2, r2 = random_pair("f64", 500_000, seed=778, rate=0.0)
+        o2[[5, 99_999, 400_000]] += 1.0
+        reps = [pin(mr), pin(1000)]
+        res = av.prepare_batch([(out, ref, 1e-6, 1e-5, mr), (o2, r2, 1e-6, 1e-5, 1000)], report_buffers=reps)
+        e1 = orc.compare(out.cpu().numpy(), ref.cpu().numpy(), "f32", 1e-6, 1e-5, mr)
+        e2 = orc.compare(o2.cpu().numpy(), r2.cpu().numpy(), "f64", 1e-6, 1e-5, 1000)
+        for it in range(3):
+            for b in reps:
+                b.view(np.uint8)[:] = 0x5A
+            g1, g2 = res()
+            assert_same(g1, e1, f"batch dense it={it}")
+            assert_same(g2, e2, f"batch sparse it={it}")

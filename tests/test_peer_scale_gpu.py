@@ -200,3 +200,76 @@ def test_sharded_north_star_shapes_nccl_two_gpus():
     for name, reps in (("C5", range(6)), ("C4", range(4))):
         for rep in reps:
             assert res[0][(name, rep)] == want[name], (name, rep)
+
+
+def _multi_worker(rank, world, port, q, n, mr):
+    sys.path.insert(0, ROOT)
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    out = []
+    try:
+        import paper_conf_ipps_leelv14_b200 as av
+
+        torch.cuda.set_device(0)
+        assert av.init_distributed(transport="peer", max_report_cap=MR) == "peer"
+        reg = synth.C5(n)
+        # ragged shards: rank r gets a slightly different length
+        cuts = [0] + [min(n, (r + 1) * n // world + 777 * (r + 1)) for r in range(world - 1)] + [n]
+        o, r = reg.slice(cuts[rank], cuts[rank + 1] - cuts[rank], device="cuda")
+        dev_rep = torch.empty(24 * MR, dtype=torch.uint8, device="cuda")
+        av.arc_verify_peer_stats(reset=True)
+        for rep in range(3):
+            g = av.compare(o, r, 0, 0, mr, report=(None, dev_rep, None)[rep])
+            out.append(((rep,), _digest(g, av)))
+        out.append((("bytes",), av.arc_verify_peer_stats()))
+        av.finalize()
+        q.put((rank, out, None))
+    except Exception:  # pragma: no cover
+        import traceback
+
+        q.put((rank, out, traceback.format_exc()))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.timeout(900)
+@pytest.mark.parametrize("world", [3, 5])
+def test_ring_many_contributors_ragged(world):
+    """Ring forwarding with several contributing ranks: C5-shaped int32 (50 % mismatches)
+    over n = 2^21 + 12345 elements in ragged shards and max_report = 2^20 - 7, so most ranks
+    contribute, contributions are not multiples of the 384 KB chunk and the last one is
+    truncated.  Every rank bit-exact against the unsharded oracle; the bytes each rank read
+    from peer windows equal (p - 1) x the report -- no window is read twice per call."""
+    import oracle
+
+    oracle.build()
+    n, mr = (1 << 21) + 12345, MR - 7
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_multi_worker, args=(r, world, port, q, n, mr)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = {}
+    try:
+        for _ in range(world):
+            rank, out, err = q.get(timeout=800)
+            assert err is None, f"rank {rank}:\n{err}"
+            res[rank] = dict(out)
+    finally:
+        for p in procs:
+            p.join(timeout=120)
+            if p.is_alive():
+                p.kill()
+    o, r = synth.C5(n).slice()
+    e = oracle.compare(o.numpy(), r.numpy(), "i32", 0, 0, mr)
+    want = (e.n, e.n_mismatch, _bits(e.max_abs_err), _bits(e.max_rel_err), e.n_reported,
+            hashlib.sha256(np.ascontiguousarray(e.report).tobytes()).hexdigest())
+    assert e.n_reported == mr
+    for rank in range(world):
+        for rep in range(3):
+            assert res[rank][(rep,)] == want, (world, rank, rep)
+    # each rank receives the report entries it does not own exactly once per call
+    # (ring: from its predecessor; its own from its own window, locally)
+    tot = sum(sum(res[rank][("bytes",)]) for rank in range(world))
+    assert tot == 3 * (world - 1) * 24 * mr, (tot, [res[k][("bytes",)] for k in range(world)])
