@@ -1549,10 +1549,18 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
             consumer_bar();
             // The CTA that arrives last has seen every count: with no tile to
             // report (the common, clean call) the results are final now, so it
-            // publishes at once instead of after the report phase's own round
-            // (which then only keeps the counter contract).
-            if (s_last && p.finalize && *(volatile uint32_t *)p.nz_cnt == 0u)
-                publish(p, ctid, kConsumerThreads, false);  // no report entry written anywhere
+            // publishes at once, and no CTA runs the report phase -- each only
+            // keeps its counter contract (one grid-barrier arrival, and with
+            // `finalize` one done arrival) with fire-and-forget reductions.
+            if (*(volatile uint32_t *)p.nz_cnt == 0u) {
+                if (s_last && p.finalize) publish(p, ctid, kConsumerThreads, false);  // no entry written anywhere
+                if (ctid == 0) {
+                    asm volatile("red.relaxed.gpu.global.add.u64 [%0], 1;" ::"l"(p.gbar) : "memory");
+                    if (p.finalize) asm volatile("red.relaxed.gpu.global.add.u64 [%0], 1;" ::"l"(p.done) : "memory");
+                }
+                if (p.xfused) exchange_tail(p, ctid, s_last != 0, smem);  // the leader published the mirror
+                return;
+            }
             report_phase(p, segs, smem, ctid, p.done_base + gridDim.x, true);
             return;
         }

@@ -277,3 +277,81 @@ def test_checksum_between_sharded_compares(fused, monkeypatch):
         for x in res[rank]:
             if x[0] == "sum":
                 assert (x[2], x[3]) == sums, (rank, x[1])
+
+
+def _clean_worker(rank, world, port, q):
+    sys.path.insert(0, ROOT)
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    out = []
+    try:
+        import paper_conf_ipps_leelv14_b200 as av
+
+        torch.cuda.set_device(0)
+        assert av.init_distributed(transport="peer", max_report_cap=1 << 12) == "peer"
+        reg = synth.C2("A")  # clean everywhere: every rank takes the no-report shortcut
+        n = 1 << 22
+        a, b = rank * n // world, (rank + 1) * n // world
+        o, r = reg.slice(a, b - a, device="cuda")
+        dirty = synth.C4(1 << 20)  # rank 0 dirty, the others clean
+        if rank == 0:
+            od, rd = dirty.slice(device="cuda")
+        else:
+            od, rd = dirty.slice(0, 1 << 18, device="cuda")
+            od = rd.clone()
+        for it in range(4):
+            g = av.compare(o, r, reg.abs_tol, reg.rel_tol, 100)
+            out.append(("clean", it, g.n, g.n_mismatch, _bits(g.max_abs_err), _bits(g.max_rel_err), g.n_reported))
+            g = av.compare(od, rd, dirty.abs_tol, dirty.rel_tol, 100)
+            out.append(("mixed", it, g.n, g.n_mismatch, g.n_reported,
+                        tuple(int(i) for i in np.asarray(g.report["index"][: g.n_reported]))))
+        av.finalize()
+        q.put((rank, out, None))
+    except Exception:  # pragma: no cover
+        import traceback
+
+        q.put((rank, out, traceback.format_exc()))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.timeout(600)
+@pytest.mark.parametrize("fused", ["1", "0"])
+def test_clean_shards_shortcut(fused, monkeypatch):
+    """Shards without a single mismatch skip the report phase (the last CTA at the grid
+    barrier publishes, the others only keep their counter contract) and still run the
+    exchange: all-clean calls and calls where only rank 0 has mismatches, alternating,
+    equal to the unsharded oracle / the generator's closed form on every rank."""
+    import oracle
+
+    oracle.build()
+    monkeypatch.setenv("ARCV_FUSED_EXCHANGE", fused)
+    world = 3
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_clean_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = {}
+    for _ in range(world):
+        rank, out, err = q.get(timeout=540)
+        assert err is None, f"rank {rank}:\n{err}"
+        res[rank] = out
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for r in range(1, world):
+        assert res[r] == res[0]
+    reg = synth.C2("A")
+    o, r = reg.slice(0, 1 << 22)
+    e = oracle.compare(o.numpy(), r.numpy(), "f32", reg.abs_tol, reg.rel_tol, 100)
+    dirty = synth.C4(1 << 20)
+    planted = dirty.planted()
+    for x in res[0]:
+        if x[0] == "clean":
+            assert x[2:] == (e.n, e.n_mismatch, _bits(e.max_abs_err), _bits(e.max_rel_err), e.n_reported)
+            assert e.n_mismatch == 0
+        else:
+            assert x[2] == (1 << 20) + 2 * (1 << 18) and x[3] == len(planted)
+            assert list(x[5]) == planted[:100]

@@ -54,9 +54,33 @@ def run(name, o, r, at, rt, mr):
                 print(f"  {kn} {nm:18s} min {d.min():8.2f}  med {np.median(d):8.2f}  max {d.max():8.2f}  (n={len(col)})")
 
 
+def run_probe(name, o, r):
+    """The read probe (same K1 pipeline, predicate off) traced like a compare."""
+    buf = np.zeros((3, 1024, 32), dtype=np.uint64)
+    lib.arc_verify_probe_read.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int,
+                                          ctypes.POINTER(ctypes.c_double)]
+    g = ctypes.c_double()
+    lib.arc_verify_probe_read(o.data_ptr(), r.data_ptr(), o.numel() * o.element_size(), 3, ctypes.byref(g))
+    lib.arc_verify_debug_trace(buf.ctypes.data_as(ctypes.POINTER(ctypes.c_ulonglong)))  # clear
+    assert lib.arc_verify_probe_read(o.data_ptr(), r.data_ptr(), o.numel() * o.element_size(), 1,
+                                     ctypes.byref(g)) == 0
+    assert lib.arc_verify_debug_trace(buf.ctypes.data_as(ctypes.POINTER(ctypes.c_ulonglong))) == 0
+    t = buf.astype(np.float64)
+    k1 = t[0][t[0][:, 0] > 0]
+    t0 = k1[:, 0].min()
+    print(f"== {name}: {len(k1)} K1 CTAs (probe: {g.value:.0f} GB/s event-timed)")
+    for i, nm in enumerate(K1):
+        col = k1[:, i]
+        col = col[col > 0]
+        if len(col):
+            d = (col - t0) / 1e3
+            print(f"  K1 {nm:18s} min {d.min():8.2f}  med {np.median(d):8.2f}  max {d.max():8.2f}  (n={len(col)})")
+
+
 if os.environ.get("TRACE_C2A"):
     c2 = synth.C2("A")
     o, r = c2.slice(device="cuda")
+    run_probe("read probe over the C2A arrays", o, r)
     run("C2A fp32 8192^2, max_report 2^20", o, r, c2.abs_tol, c2.rel_tol, c2.max_report)
     run("C2A fp32 8192^2, count only", o, r, c2.abs_tol, c2.rel_tol, 0)
     run("C2A bytes as u8 (no float filter), count only", o.view(torch.uint8), r.view(torch.uint8), 0, 0, 0)
