@@ -232,7 +232,9 @@ uint64_t arc_verify_launch_count(void);
  * stream two device buffers of `bytes` each through the same bulk-copy pipeline
  * as the comparison, with the predicate disabled, `iters` times, and return the
  * achieved read bandwidth in GB/s (2 * bytes * iters / time).  It is the in-run
- * read-only ceiling the comparison kernel is judged against.
+ * read-only ceiling the comparison kernel is judged against.  Each launch is
+ * timed on its own from an idle stream (CUDA events around the launch), as a
+ * compare call runs and as arc_verify_kernel_stats times it.
  * Errors: ARC_E_INVAL (NULL / host buffers, bytes == 0, iters < 1), ARC_E_NOINIT.
  */
 int arc_verify_probe_read(const void *a, const void *b, uint64_t bytes, int iters, double *gbs);

@@ -1335,7 +1335,10 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
     if (p.finalize) {
         const bool last = last_cta(p, tid, kConsumerThreads, &sh.last, wrote_host, done_base);
         if (tid == 0) ARCV_STAMP(1, 11);
-        if (last && !(k1_published_if_empty && n_nz == 0)) publish(p, tid, kConsumerThreads);
+        // a report kept in device memory (the caller's buffer or HBM staging that
+        // the host copies later, stream-ordered) needs no system fence before the
+        // completion word: the slots validate themselves (slot_tag)
+        if (last && !(k1_published_if_empty && n_nz == 0)) publish(p, tid, kConsumerThreads, p.report_host != 0);
         if (p.xfused) exchange_tail(p, tid, last, smem);
     }
     if (tid == 0) ARCV_STAMP(1, 7);
