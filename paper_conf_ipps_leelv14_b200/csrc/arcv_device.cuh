@@ -303,23 +303,48 @@ __device__ __forceinline__ void share_bounds(ThreadAcc &acc) {
 // with near-final bounds instead of flagging every record-breaking element.
 // Evaluating an element here and again in the main pass is harmless: maxima
 // are idempotent and the mismatch decision is taken by the main pass.
-template <typename T>
+template <typename T, bool kAligned>
 __device__ __forceinline__ void seed_bounds(const uint8_t *so, const uint8_t *sr, uint32_t off_o, uint32_t off_r,
                                             uint32_t cnt, int ctid, const SegHot &g, ThreadAcc &acc) {
     constexpr int EPV = 16 / sizeof(T);
     acc.seeded = true;
     float best_d = -1.f, best_r = -1.f;
     int bd = -1, br = -1;
-    ARCV_UNROLL(ARCV_SEED_UNROLL)
-    for (int b = 0; b < kVecPerThread * EPV; ++b) {
-        const uint32_t e = (uint32_t)(((b / EPV) * kConsumerThreads + ctid) * EPV + (b % EPV));
-        if (e >= cnt) continue;
-        const T x = *reinterpret_cast<const T *>(so + off_o + e * sizeof(T));
-        const T y = *reinterpret_cast<const T *>(sr + off_r + e * sizeof(T));
-        const float d = (float)fabs((double)x - (double)y);
-        const float r = __fdividef(d, fabsf((float)y) + 1e-37f);
-        if (d > best_d && d < CUDART_INF_F) { best_d = d; bd = b; }
-        if (r > best_r && r < CUDART_INF_F) { best_r = r; br = b; }
+    // The scan only picks which two elements to evaluate exactly, so it may be
+    // approximate: fp32 arithmetic for fp32 data (no fp64 conversions), 16-byte
+    // vector loads when the tile is aligned (profiles: the first tile of a
+    // float region is issue-bound on this scan).
+    ARCV_UNROLL(ARCV_EVAL_UNROLL)
+    for (int k = 0; k < kVecPerThread; ++k) {
+        const uint32_t v = k * kConsumerThreads + ctid;
+        T xo[EPV], xr[EPV];
+        if constexpr (kAligned) {
+            const uint4 a = reinterpret_cast<const uint4 *>(so)[v];
+            const uint4 c = reinterpret_cast<const uint4 *>(sr)[v];
+            memcpy(xo, &a, 16);
+            memcpy(xr, &c, 16);
+        } else {
+#pragma unroll
+            for (int j = 0; j < EPV; ++j) {
+                xo[j] = *reinterpret_cast<const T *>(so + off_o + (v * EPV + j) * sizeof(T));
+                xr[j] = *reinterpret_cast<const T *>(sr + off_r + (v * EPV + j) * sizeof(T));
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < EPV; ++j) {
+            if (v * EPV + j >= cnt) continue;
+            float d, r;
+            if constexpr (std::is_same<T, float>::value) {
+                d = fabsf(__fsub_rn(xo[j], xr[j]));
+                r = __fdividef(d, fabsf(xr[j]) + 1e-37f);
+            } else {
+                d = (float)fabs(xo[j] - xr[j]);
+                r = __fdividef(d, fabsf((float)xr[j]) + 1e-37f);
+            }
+            const int b = k * EPV + j;
+            if (d > best_d && d < CUDART_INF_F) { best_d = d; bd = b; }
+            if (r > best_r && r < CUDART_INF_F) { best_r = r; br = b; }
+        }
     }
     for (int q = 0; q < 2; ++q) {
         const int b = q == 0 ? bd : br;
@@ -351,7 +376,7 @@ __device__ __forceinline__ uint32_t eval_tile(const uint8_t *so, const uint8_t *
     bool rel_form = true;
     if constexpr (kFloat) {
         if (!acc.seeded) {
-            seed_bounds<T>(so, sr, off_o, off_r, cnt, ctid, g, acc);
+            seed_bounds<T, kAligned>(so, sr, off_o, off_r, cnt, ctid, g, acc);
             share_bounds(acc);
 #if !defined(ARCV_BLOCK_SEED) || ARCV_BLOCK_SEED
             // block-wide: every consumer warp seeds on this same tile (all
