@@ -312,8 +312,22 @@ __device__ __forceinline__ void seed_bounds(const uint8_t *so, const uint8_t *sr
     int bd = -1, br = -1;
     // The scan only picks which two elements to evaluate exactly, so it may be
     // approximate: fp32 arithmetic for fp32 data (no fp64 conversions), 16-byte
-    // vector loads when the tile is aligned (profiles: the first tile of a
-    // float region is issue-bound on this scan).
+    // vector loads when the tile is aligned (f32x12 113.2 -> 110.9 us,
+    // profiles/r02x_ab_seed_scan_fp32.log).  fp64 data keeps the plain scalar
+    // scan (no gain there; its variants stay unchanged).
+    if constexpr (!std::is_same<T, float>::value) {
+        ARCV_UNROLL(ARCV_SEED_UNROLL)
+        for (int b = 0; b < kVecPerThread * EPV; ++b) {
+            const uint32_t e = (uint32_t)(((b / EPV) * kConsumerThreads + ctid) * EPV + (b % EPV));
+            if (e >= cnt) continue;
+            const T x = *reinterpret_cast<const T *>(so + off_o + e * sizeof(T));
+            const T y = *reinterpret_cast<const T *>(sr + off_r + e * sizeof(T));
+            const float d = (float)fabs((double)x - (double)y);
+            const float r = __fdividef(d, fabsf((float)y) + 1e-37f);
+            if (d > best_d && d < CUDART_INF_F) { best_d = d; bd = b; }
+            if (r > best_r && r < CUDART_INF_F) { best_r = r; br = b; }
+        }
+    } else {
     ARCV_UNROLL(ARCV_EVAL_UNROLL)
     for (int k = 0; k < kVecPerThread; ++k) {
         const uint32_t v = k * kConsumerThreads + ctid;
@@ -345,6 +359,7 @@ __device__ __forceinline__ void seed_bounds(const uint8_t *so, const uint8_t *sr
             if (d > best_d && d < CUDART_INF_F) { best_d = d; bd = b; }
             if (r > best_r && r < CUDART_INF_F) { best_r = r; br = b; }
         }
+    }
     }
     for (int q = 0; q < 2; ++q) {
         const int b = q == 0 ? bd : br;
