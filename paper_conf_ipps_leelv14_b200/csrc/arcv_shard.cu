@@ -84,11 +84,11 @@ static NcclApi nccl;
 
 static int load_nccl() {
     if (nccl.h) return ARC_OK;
-    void *h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);  // the copy torch already loaded
-    if (!h) {
-        const char *env = getenv("ARCV_NCCL_LIB");
-        h = dlopen(env && *env ? env : "libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
-    }
+    // ARCV_NCCL_LIB (diagnostics / tests) names the library explicitly and wins;
+    // otherwise the copy torch already loaded, else the system's.
+    const char *env = getenv("ARCV_NCCL_LIB");
+    void *h = (env && *env) ? dlopen(env, RTLD_NOW | RTLD_LOCAL) : dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
+    if (!h && !(env && *env)) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
     if (!h) {
         set_error("cannot load NCCL: %s", dlerror());
         return ARC_E_NCCL;
