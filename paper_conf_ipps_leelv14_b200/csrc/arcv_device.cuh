@@ -1102,13 +1102,11 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
     // library's staging for a pageable buffer) gets its entries written there
     // directly over PCIe when direct_route() holds -- K1's final count and the
     // path taken decide it; the host applies the same rule to the published
-    // slot.  `tc` = the tile's count (pool path; 0 if unknown), `part` / `S`:
-    // this CTA writes in-tile ranks [part * ceil(tc / S), ...) only (a dense
-    // tile split across S CTAs); split or dense direct tiles go through the
-    // shared-memory out buffer (coalesced stores).
+    // slot.  `tc` = the tile's count (pool path; 0 if unknown): a dense tile
+    // going straight to pinned memory is written through the shared-memory out
+    // buffer as coalesced words.
     arc_mismatch_t *const obuf = reinterpret_cast<arc_mismatch_t *>(smem + 2 * kStageBytes + sizeof(RepShared));
-    auto emit = [&](uint64_t key, uint64_t excl, int st, bool pool, uint64_t tc, uint32_t part, uint32_t S,
-                    bool stamp = false) {
+    auto emit = [&](uint64_t key, uint64_t excl, int st, bool pool, uint64_t tc, bool stamp = false) {
         const Seg &g = segs[key >> 40];
         const bool direct = direct_route(g.report_alias != nullptr, g.flags, __ldcg(&p.acc[g.acc_slot].count),
                                          g.max_report, g.alias_cap, pool);
@@ -1124,38 +1122,26 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
             const uint8_t *so = smem + (size_t)st * kStageBytes;
             const uint64_t mask = mask_any(so, so + kStageArrayBytes, si, tid, g);
             if (tid == 0 && stamp) ARCV_STAMP(1, 5);
-            const bool staged = S > 1 || (direct && tc > kStagedMin);
-            const uint64_t per = (tc + S - 1) / S;
-            const uint64_t rlo = staged ? (uint64_t)part * per : 0ull;
-            const uint64_t rhi = staged ? (rlo + per < tc ? rlo + per : tc) : ~0ull;
+            const bool staged = direct && tc > kStagedMin;
             compact_any(g, si, so, so + kStageArrayBytes, mask, excl | (direct ? kDirectBit : 0ull), sh.w, tid,
-                        rlo, rhi, staged ? obuf : nullptr);
+                        0ull, staged ? tc : ~0ull, staged ? obuf : nullptr);
         }
         consumer_bar();  // stage `st` and sh.w are reused
         if (tid == 0 && stamp) ARCV_STAMP(1, 2);
     };
 
     const uint32_t n_nz = *(volatile uint32_t *)p.nz_cnt;
-    // the reporting regions' final counts (the pool path's split decision),
-    // loaded alongside n_nz: no extra round trip on the critical path
-    uint64_t tot_cnt = 0;
-    if (p.n_segs <= (uint32_t)kMaxInlineSegs)
-        for (uint32_t sgi = 0; sgi < p.n_segs; ++sgi)
-            if (segs[sgi].max_report) tot_cnt += __ldcg(&p.acc[segs[sgi].acc_slot].count);
     const uint32_t G = gridDim.x, b = blockIdx.x;
     if (n_nz <= (uint32_t)kPoolCap) {
         // ------------------------------------------------------ pool path
         // arrive on the grid-barrier counter without waiting (host base += grid)
         if (tid == 0) atomicAdd(p.gbar, 1ull);
-        // few listed tiles that are dense on average (> kStagedMin mismatches per
-        // tile): each is split across S CTAs, so a dense tile's entries are
-        // written by S SMs; work item i = pool entry i / S, part i % S.  Every
-        // CTA derives the same S from the final counts.
-        uint32_t S = 1u;
-        if (n_nz > 0 && 2 * n_nz <= G && p.n_segs <= (uint32_t)kMaxInlineSegs &&
-            tot_cnt > (uint64_t)n_nz * kStagedMin)
-            S = min(kSplitMax, G / n_nz);
-        const uint32_t n_items = n_nz * S;
+        // (Round 2 measured splitting a dense tile across several CTAs: C2B
+        // -10 us per call, but any form of that code in K1's tail -- inline or
+        // out of line -- changed the stream loop's code generation and cost
+        // sparse calls ~2 us and C3 ~5 us (profiles/r02ah_ab.log,
+        // r02aj_ab.log); dense direct tiles are written by one CTA, staged.)
+        const uint32_t n_items = n_nz;
 #if defined(ARCV_TAIL_REPS)
       // diagnostic: run the (idempotent) pool path again, stamps from the last run
       for (int rep_ = 0; rep_ < ARCV_TAIL_REPS; ++rep_) {
@@ -1163,7 +1149,7 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
         if (tid == 0) ARCV_STAMP(1, 8);
 #endif
         const uint32_t n_own = n_items > b ? (n_items - b + G - 1) / G : 0u;
-        auto entry_of = [&](uint32_t j) { return (b + j * G) / S; };  // my j-th item's pool entry
+        auto entry_of = [&](uint32_t j) { return b + j * G; };  // my j-th pool entry
         const ulonglong2 *nzl = reinterpret_cast<const ulonglong2 *>(p.nz_list);
         // One round trip for everything the prefixes and the first re-reads
         // need: the CTA's first two pool entries (every thread: they are also
@@ -1193,14 +1179,12 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
         for (uint32_t j0 = 0; j0 < n_own; j0 += 2) {
             const uint32_t m = n_own - j0 < 2u ? n_own - j0 : 2u;
             uint64_t key[2], tcn[2] = {0, 0}, pre[2] = {0, 0}, tot[2] = {0, 0};
-            uint32_t part[2] = {0, 0};
 #pragma unroll
             for (int q = 0; q < 2; ++q) {
                 if ((uint32_t)q < m) {
                     const ulonglong2 e = j0 == 0 ? kv[q] : __ldcg(nzl + entry_of(j0 + q));
                     key[q] = e.x;
                     tcn[q] = e.y;
-                    part[q] = (b + (j0 + q) * G) % S;
                 } else {
                     key[q] = ~0ull - 1;
                 }
@@ -1232,7 +1216,7 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
                 for (int c = 0; c < 4; ++c) r[c] += sh.red[w][c];
             if (tid == 0) ARCV_STAMP(1, 3);
 #if !defined(ARCV_HALF_TILES) || ARCV_HALF_TILES
-            bool half = m == 2 && S == 1 && segs[key[0] >> 40].dtype != ARC_U8 && segs[key[1] >> 40].dtype != ARC_U8;
+            bool half = m == 2 && segs[key[0] >> 40].dtype != ARC_U8 && segs[key[1] >> 40].dtype != ARC_U8;
             if (half) {  // not for dense tiles going straight to pinned memory (staged writes)
 #pragma unroll
                 for (int q = 0; q < 2; ++q) {
@@ -1281,8 +1265,8 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
                 const uint64_t seg_tot = r[2 + q];
                 uint64_t base = 0;
                 if (g.flags & kSegBaseFromAcc) base = __ldcg(&p.acc[g.acc_slot].count) - seg_tot;
-                if (tid == 0 && part[q] == 0) p.tile_cnt[g.slot_begin + (key[q] & kLtMask)] = 0u;  // clean
-                emit(key[q], base + r[q], q, true, tcn[q], part[q], S, j == 0);  // ends with a barrier
+                if (tid == 0) p.tile_cnt[g.slot_begin + (key[q] & kLtMask)] = 0u;  // clean for the next call
+                emit(key[q], base + r[q], q, true, tcn[q], j == 0);  // ends with a barrier
                 if (tid == 0 && j == 1) ARCV_STAMP(1, 10);
                 if (tid == 0 && j + 2 < n_own) issue(__ldcg(p.nz_list + 2 * entry_of(j + 2)), q);
             }
@@ -1357,7 +1341,7 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
             if (j + 1 < mine && tid == 0) issue(__ldcg(p.active + 2 * (b + (j + 1) * G)), st ^ 1);  // prefetch
             const uint64_t key = __ldcg(p.active + 2 * (b + j * G));
             const uint64_t excl = __ldcg(p.active + 2 * (b + j * G) + 1);
-            emit(key, excl, st, false, 0, 0, 1);
+            emit(key, excl, st, false, 0);
         }
     }
     // Report entries in pinned host memory need no system-scope fence here:

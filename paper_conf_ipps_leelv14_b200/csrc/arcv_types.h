@@ -23,11 +23,10 @@ constexpr int kPoolCap = 2048;                      // report phase, pool path: 
 constexpr uint64_t kDirectDyn = ARCV_DIRECT_DYN;               // sparse reports: written directly into pinned host memory
 constexpr uint64_t kDirectBit = 1ull << 63;         // report-phase tile prefix flag: entries go to report_alias
 // Pool path (<= kPoolCap reported tiles): a denser pinned-host report is still
-// written by the kernel itself, staged per CTA in shared memory and stored as
-// coalesced 8-byte words from many CTAs (a dense tile is split across up to
-// kSplitMax CTAs), up to kDirectDense entries; beyond that HBM staging + one D2H.
+// written by the kernel itself, each dense tile staged in shared memory and
+// stored as coalesced 8-byte words, up to kDirectDense entries; beyond that
+// HBM staging + one D2H.
 constexpr uint64_t kDirectDense = 1ull << 18;
-constexpr uint32_t kSplitMax = 16;
 constexpr uint64_t kStagedMin = 64;                 // tiles with more entries: staged, coalesced writes
 constexpr uint64_t kPinStage = 1ull << 16;          // pageable report: library pinned staging per region
 constexpr uint64_t kRoutePool = 1ull;               // Acc.pad of a published slot: the report took the pool path

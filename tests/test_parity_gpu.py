@@ -787,23 +787,23 @@ def test_env_flags_cannot_disable_the_predicate():
 
 
 @pytest.mark.parametrize("dt,n_dense,mr,buf,off", [
-    ("f32", 2, 1 << 20, "pinned", 0),      # C2B-like: 2 dense tiles, split across CTAs, direct
+    ("f32", 2, 1 << 20, "pinned", 0),      # C2B-like: 2 dense tiles, staged coalesced direct writes
     ("f32", 2, 1 << 20, "pageable", 1),    # library pinned staging, misaligned arrays
     ("f32", 2, 5000, "pinned", 0),         # truncation inside the second tile
     ("f64", 20, 1 << 20, "pinned", 0),     # 40960 entries, pool path, direct
     ("f64", 20, 1 << 20, "pageable", 0),   # > the 2^16 pageable staging: HBM staging + D2H
     ("i32", 100, 1 << 20, "pinned", 3),    # 409600 > 2^18 entries: HBM staging + D2H
     ("i32", 100, 7777, "pinned", 0),       # truncated far below: direct
-    ("u8", 3, 1 << 20, "pinned", 5),       # u8 tiles (16384 elements), split
-    ("f32", 2, 1 << 20, "device", 0),      # device report: split tiles, staged coalesced stores
-    ("f32", 1, 1 << 20, "pinned", 0),      # one dense tile split across up to 16 CTAs
+    ("u8", 3, 1 << 20, "pinned", 5),       # u8 tiles (16384 elements), several staging rounds
+    ("f32", 2, 1 << 20, "device", 0),      # device report: plain scattered stores
+    ("f32", 1, 1 << 20, "pinned", 0),      # one dense tile
 ])
 def test_dense_tiles_direct_route(av, orc, dt, n_dense, mr, buf, off):
     """Few report tiles holding many mismatches (C2B's shape: a wrong loop bound leaves a
-    whole row stale): the pool path splits each dense tile across several CTAs, which write
-    their rank ranges through shared memory as coalesced words -- into the caller's pinned
-    buffer (or the library's pinned staging) when direct_route() allows, else into HBM
-    staging followed by one D2H copy.  Every combination bit-exact against the oracle."""
+    whole row stale): the pool path writes a dense tile's entries through shared memory as
+    coalesced words (in rounds of 1024 entries) -- into the caller's pinned buffer (or the
+    library's pinned staging) when direct_route() allows, else into HBM staging followed by
+    one D2H copy.  Every combination bit-exact against the oracle."""
     te = TILE_ELEMS[dt]
     n = te * (n_dense * 3 + 5) + 123
     out, ref = random_pair(dt, n + off, seed=4242 + n_dense, rate=0.0)
@@ -830,7 +830,7 @@ def test_dense_tiles_direct_route(av, orc, dt, n_dense, mr, buf, off):
 
 @pytest.mark.parametrize("kind", ["checks", "batch"])
 def test_dense_tiles_checks_and_batches(av, orc, kind):
-    """The split / staged dense-tile route combined with the N2 checks (minValueToCheck and
+    """The staged dense-tile route combined with the N2 checks (minValueToCheck and
     value bounds remove some mismatches inside the dense tiles, so K1's counts and the
     report phase's ranks must agree under the checks) and inside a batch (a dense region
     and a sparse one sharing the pool, each with its own pinned report)."""
