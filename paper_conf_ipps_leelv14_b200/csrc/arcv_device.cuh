@@ -1072,6 +1072,7 @@ struct RepShared {
 // [stage 0][stage 1][RepShared][out buffer: kOutEntries entries]
 constexpr int kReportSmem = 2 * kStageBytes + (int)sizeof(RepShared) + kOutEntries * (int)sizeof(arc_mismatch_t);
 
+template <bool XF>
 __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, uint8_t *smem, int tid,
                                              unsigned long long done_base, bool k1_published_if_empty) {
     RepShared &sh = *reinterpret_cast<RepShared *>(smem + 2 * kStageBytes);
@@ -1363,7 +1364,9 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
         // the host copies later, stream-ordered) needs no system fence before the
         // completion word: the slots validate themselves (slot_tag)
         if (last && !(k1_published_if_empty && n_nz == 0)) publish(p, tid, kConsumerThreads, p.report_host != 0);
-        if (p.xfused) exchange_tail(p, tid, last, smem);
+        if constexpr (XF) {
+            if (p.xfused) exchange_tail(p, tid, last, smem);
+        }
     }
     if (tid == 0) ARCV_STAMP(1, 7);
 }
@@ -1382,12 +1385,14 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
     // touching any of them
     asm volatile("griddepcontrol.wait;" ::: "memory");
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");  // the exchange kernel, if any
-    report_phase(p, segs, smem, (int)threadIdx.x, p.done_base, true);
+    report_phase<false>(p, segs, smem, (int)threadIdx.x, p.done_base, true);
 }
 
 
 // ------------------------------------------------------------------ K1: stream
-template <int S, int MINB, int NSEG>
+// XF: the sharded exchange is fused into this kernel's tail (its own
+// instantiation, so single-GPU calls carry none of the exchange code).
+template <int S, int MINB, int NSEG, bool XF = false>
 __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __grid_constant__ ParamsN<NSEG> pn) {
     const Params &p = pn;
     extern __shared__ __align__(128) uint8_t smem[];
@@ -1585,10 +1590,12 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
                     asm volatile("red.relaxed.gpu.global.add.u64 [%0], 1;" ::"l"(p.gbar) : "memory");
                     if (p.finalize) asm volatile("red.relaxed.gpu.global.add.u64 [%0], 1;" ::"l"(p.done) : "memory");
                 }
-                if (p.xfused) exchange_tail(p, ctid, s_last != 0, smem);  // the leader published the mirror
+                if constexpr (XF) {
+                    if (p.xfused) exchange_tail(p, ctid, s_last != 0, smem);  // the leader published the mirror
+                }
                 return;
             }
-            report_phase(p, segs, smem, ctid, p.done_base + gridDim.x, true);
+            report_phase<XF>(p, segs, smem, ctid, p.done_base + gridDim.x, true);
             return;
         }
     }
@@ -1600,7 +1607,9 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
         if (p.finalize && (!p.k2 || *(volatile uint32_t *)p.nz_cnt == 0u))
             publish(p, ctid, kConsumerThreads, false);  // count-only / clean: no report entry written
     }
-    if (p.xfused) exchange_tail(p, ctid, s_last != 0, smem);  // count-only sharded call (no K2 then)
+    if constexpr (XF) {
+        if (p.xfused) exchange_tail(p, ctid, s_last != 0, smem);  // count-only sharded call (no K2 then)
+    }
     if (ctid == 0) ARCV_STAMP(0, 3);
 }
 

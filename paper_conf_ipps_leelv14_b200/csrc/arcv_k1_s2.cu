@@ -11,5 +11,6 @@ namespace arcv {
 
 KernelFnN<1> k1_s2_1() { return arcv_stream_kernel<2, 3, 1>; }
 KernelFnN<kMaxInlineSegs> k1_s2_n() { return arcv_stream_kernel<2, 3, kMaxInlineSegs>; }
+KernelFnN<1> k1_s2_1x() { return arcv_stream_kernel<2, 3, 1, true>; }  // sharded: exchange fused
 
 }  // namespace arcv

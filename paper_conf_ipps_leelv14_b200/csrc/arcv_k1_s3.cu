@@ -11,6 +11,7 @@ namespace arcv {
 
 KernelFnN<1> k1_s3_1() { return arcv_stream_kernel<3, 2, 1>; }
 KernelFnN<kMaxInlineSegs> k1_s3_n() { return arcv_stream_kernel<3, 2, kMaxInlineSegs>; }
+KernelFnN<1> k1_s3_1x() { return arcv_stream_kernel<3, 2, 1, true>; }  // sharded: exchange fused
 
 // K2: the separate report kernel (used with S = 2 K1s or ARCV_FUSED=0)
 KernelFnN<1> k2_fn_1() { return arcv_compact_kernel<1>; }

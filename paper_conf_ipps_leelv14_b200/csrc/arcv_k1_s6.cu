@@ -11,5 +11,6 @@ namespace arcv {
 
 KernelFnN<1> k1_s6_1() { return arcv_stream_kernel<6, 1, 1>; }
 KernelFnN<kMaxInlineSegs> k1_s6_n() { return arcv_stream_kernel<6, 1, kMaxInlineSegs>; }
+KernelFnN<1> k1_s6_1x() { return arcv_stream_kernel<6, 1, 1, true>; }  // sharded: exchange fused
 
 }  // namespace arcv

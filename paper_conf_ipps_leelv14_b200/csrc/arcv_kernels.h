@@ -12,12 +12,14 @@ namespace arcv {
 template <int NSEG>
 using KernelFnN = void (*)(ParamsN<NSEG>);
 
-// K1 with S stages (S in {2, 3, 4, 6}); nullptr for other S.
-KernelFnN<1> k1_fn_1(int stages);
+// K1 with S stages (S in {2, 3, 4, 6}); `xf`: the variant with the sharded
+// exchange fused into its tail (single-segment parameter blocks only).
+KernelFnN<1> k1_fn_1(int stages, bool xf = false);
 KernelFnN<kMaxInlineSegs> k1_fn_n(int stages);
 // per-TU providers (arcv_k1_s<S>.cu)
 #define ARCV_K1_DECL(S)                    \
     KernelFnN<1> k1_s##S##_1();            \
+    KernelFnN<1> k1_s##S##_1x();           \
     KernelFnN<kMaxInlineSegs> k1_s##S##_n();
 ARCV_K1_DECL(2)
 ARCV_K1_DECL(3)
