@@ -860,3 +860,45 @@ def test_dense_tiles_checks_and_batches(av, orc, kind):
             g1, g2 = res()
             assert_same(g1, e1, f"batch dense it={it}")
             assert_same(g2, e2, f"batch sparse it={it}")
+
+
+# ------------------------------------- clustered mismatches around the pool capacity
+@pytest.mark.parametrize("dt", ["f32", "f64", "i32", "i64", "u8"])
+@pytest.mark.parametrize("n_mis", [1, 700, 2047, 2048, 2049, 2600])
+def test_clustered_mismatches_reuse_tiles(av, orc, dt, n_mis):
+    """1 .. 2600 mismatches clustered in six tiles (hundreds per tile: pool path, several
+    mismatches per thread, ranks across warps and vectors) plus one in the ragged tail tile,
+    every dtype.  Each config alternates with a dense call over the SAME tiles (the report phase
+    must leave the per-tile counts clean for the next call), with several truncations, a device
+    report, and a two-region batch over overlapping views."""
+    te = TILE_ELEMS[dt]
+    n = 64 * te + 333
+    gen = torch.Generator(device="cpu").manual_seed(9100 + n_mis)
+    idx = torch.randperm(6 * te, generator=gen)[:n_mis] + 5 * te  # tiles 5..10: several per tile
+    idx[0] = n - 1  # and one in the ragged tail tile
+    if dt in ("f32", "f64"):
+        ref = (torch.rand(n, generator=gen, dtype=torch.float64) + 0.5).to(TD[dt])
+        out = ref.clone()
+        out[idx] = out[idx] * 1.5
+    else:
+        hi = 200 if dt == "u8" else 1 << 30
+        ref = torch.randint(0, hi, (n,), generator=gen).to(TD[dt])
+        out = ref.clone()
+        out[idx] = out[idx] + 7
+    dense = ref.clone()
+    dense[5 * te: 11 * te] = (dense[5 * te: 11 * te] + 3).to(TD[dt])
+    on, rn, dn = out.numpy(), ref.numpy(), dense.numpy()
+    out, ref, dense = out.cuda(), ref.cuda(), dense.cuda()
+    for mr in (1, n_mis // 2 + 1, 1 << 20):
+        e = orc.compare(on, rn, dt, 1e-6, 1e-5, mr)
+        ed = orc.compare(dn, rn, dt, 1e-6, 1e-5, mr)
+        for it in range(3):
+            assert_same(av.compare(out, ref, 1e-6, 1e-5, mr), e, f"{dt} n_mis={n_mis} mr={mr} it={it}")
+            assert_same(av.compare(dense, ref, 1e-6, 1e-5, mr), ed, f"{dt} dense mr={mr} it={it}")
+    # device report, and a batch of the sparse region with itself (two regions, one capture)
+    rep = torch.empty(24 * (1 << 20), dtype=torch.uint8, device="cuda")
+    assert_same(av.compare(out, ref, 1e-6, 1e-5, 1 << 20, report=rep), e, f"{dt} device report")
+    if n_mis <= 1024:
+        gs = av.batch([(out, ref, 1e-6, 1e-5, 1 << 20), (out[te:], ref[te:], 1e-6, 1e-5, 17)])
+        assert_same(gs[0], e, f"{dt} batch region 0")
+        assert_same(gs[1], orc.compare(on[te:], rn[te:], dt, 1e-6, 1e-5, 17), f"{dt} batch region 1")
