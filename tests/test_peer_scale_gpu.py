@@ -18,8 +18,9 @@ Report buffers: pageable host memory, pinned host memory and device memory.
 Every rank must hold the identical global result, bit-exact against the
 unsharded oracle (compare_threads: the oracle on contiguous chunks merged by
 merge_shards, pinned equal to the sequential oracle in tests/test_oracle.py).
-The second test checks the NCCL transport with two ranks on two GPUs; it skips
-on a one-GPU box (NCCL refuses two ranks on one device).
+Two more tests need one GPU per rank and skip on a one-GPU box: the peer exchange
+across 2 / 4 / 8 physical GPUs, and the NCCL transport with two ranks on two GPUs
+(NCCL refuses two ranks on one device).
 """
 import hashlib
 import os
@@ -187,6 +188,22 @@ def test_sharded_north_star_shapes_peer(world):
         for r in range(2, world):
             assert per_rank[r] == (0, rep_bytes), (r, per_rank)
     # C4 (516 entries, pull): each rank reads the other ranks' contributions once
+
+
+@pytest.mark.timeout(1500)
+@pytest.mark.parametrize("world", [2, 4, 8])
+def test_sharded_north_star_shapes_peer_own_gpus(world):
+    """The peer exchange with one rank per physical GPU (windows mapped over NVLink /
+    NVSwitch instead of within one device); skips unless `world` GPUs are visible."""
+    if torch.cuda.device_count() < world:
+        pytest.skip(f"needs {world} GPUs (one per rank); {torch.cuda.device_count()} visible")
+    res = _run(world, "peer", _own_gpu)
+    for r in range(1, world):
+        assert _results(res[r]) == _results(res[0]), f"rank {r} differs from rank 0"
+    want = _expected(world)
+    for name, reps in (("C5", range(6)), ("C4", range(4))):
+        for rep in reps:
+            assert res[0][(name, rep)] == want[name], (world, name, rep)
 
 
 @pytest.mark.timeout(1500)
