@@ -550,8 +550,16 @@ __device__ __forceinline__ uint32_t eval_tile_dispatch(const uint8_t *so, const 
     return eval_tile<T, false, false>(so, sr, si.off_o, si.off_r, si.count, ctid, g, acc);
 }
 
+// DT >= 0: a K1 specialised for one dtype (single-region calls) evaluates only
+// that dtype's tiles; DT < 0: any dtype (batches, tables).
+template <int DT = -1>
 __device__ __forceinline__ uint32_t eval_any(const uint8_t *so, const uint8_t *sr, const StageInfo &si, int ctid,
                                              const SegHot &g, ThreadAcc &acc) {
+    if constexpr (DT == ARC_F32) return eval_tile_dispatch<float>(so, sr, si, ctid, g, acc);
+    if constexpr (DT == ARC_F64) return eval_tile_dispatch<double>(so, sr, si, ctid, g, acc);
+    if constexpr (DT == ARC_I32) return eval_tile_dispatch<int32_t>(so, sr, si, ctid, g, acc);
+    if constexpr (DT == ARC_I64) return eval_tile_dispatch<int64_t>(so, sr, si, ctid, g, acc);
+    if constexpr (DT == ARC_U8) return eval_tile_dispatch<uint8_t>(so, sr, si, ctid, g, acc);
     switch (g.dtype) {
         case ARC_F32: return eval_tile_dispatch<float>(so, sr, si, ctid, g, acc);
         case ARC_F64: return eval_tile_dispatch<double>(so, sr, si, ctid, g, acc);
@@ -1392,7 +1400,7 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
 // ------------------------------------------------------------------ K1: stream
 // XF: the sharded exchange is fused into this kernel's tail (its own
 // instantiation, so single-GPU calls carry none of the exchange code).
-template <int S, int MINB, int NSEG, bool XF = false>
+template <int S, int MINB, int NSEG, bool XF = false, int DT = -1>
 __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __grid_constant__ ParamsN<NSEG> pn) {
     const Params &p = pn;
     extern __shared__ __align__(128) uint8_t smem[];
@@ -1511,7 +1519,7 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
             g.seed_sh = s_red_d;
         }
         const uint8_t *so = smem + (size_t)s * kStageBytes;
-        const uint32_t cnt = (p.flags & kFlagProbe) ? 0u : eval_any(so, so + kStageArrayBytes, si, ctid, g, acc);
+        const uint32_t cnt = (p.flags & kFlagProbe) ? 0u : eval_any<DT>(so, so + kStageArrayBytes, si, ctid, g, acc);
         acc.count += cnt;
         if (ctid == 0 && i == 0) ARCV_STAMP(0, 5);
 #if defined(ARCV_TRACE) && ARCV_TRACE

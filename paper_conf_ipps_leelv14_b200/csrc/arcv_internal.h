@@ -25,6 +25,7 @@ struct Ctx {
     uint64_t direct_max = 0;  // pinned host reports up to this capacity: written by the kernel
     bool fused = true;  // report phase in K1's tail (cooperative K1), no K2 launch
     bool pdl = true;  // launch K2 / the exchange kernel as programmatic dependents (ARCV_PDL=0: off)
+    bool dt_spec = true;  // single-region calls: K1 specialised for the region's dtype (ARCV_DT_SPEC=0: generic)
     bool sort_segs = true;  // batches: smallest regions' tiles first (ARCV_SORT_SEGS=0: listed order)
     cudaStream_t stream = nullptr;
     bool own_stream = false;

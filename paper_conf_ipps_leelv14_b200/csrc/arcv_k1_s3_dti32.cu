@@ -1,0 +1,15 @@
+// arcv_k1_s3_dti32.cu -- K1 with 3 stages, min 2 CTAs per SM, specialised for
+// ARC_I32 regions (single-region calls: only that dtype's tile evaluation is
+// compiled in, so the kernel is ~5x smaller); arcv_kernels.h.
+#include <cuda_runtime.h>
+
+#include "arcv_device.cuh"
+#include "arcv_kernels.h"
+
+namespace arcv {
+
+KernelFnN<1> k1_s3_1_i32(bool xf) {
+    return xf ? arcv_stream_kernel<3, 2, 1, true, ARC_I32> : arcv_stream_kernel<3, 2, 1, false, ARC_I32>;
+}
+
+}  // namespace arcv

@@ -26,6 +26,14 @@ ARCV_K1_DECL(3)
 ARCV_K1_DECL(4)
 ARCV_K1_DECL(6)
 #undef ARCV_K1_DECL
+// K1 with 3 stages specialised for one dtype (single-region calls; `xf` as
+// above), one translation unit per dtype (arcv_k1_s3_dt<dtype>.cu)
+KernelFnN<1> k1_s3_1_f32(bool xf);
+KernelFnN<1> k1_s3_1_f64(bool xf);
+KernelFnN<1> k1_s3_1_i32(bool xf);
+KernelFnN<1> k1_s3_1_i64(bool xf);
+KernelFnN<1> k1_s3_1_u8(bool xf);
+KernelFnN<1> k1_fn_1_dt(int stages, bool xf, int dtype);  // nullptr: no specialisation
 // K2 (arcv_k1_s3.cu)
 KernelFnN<1> k2_fn_1();
 KernelFnN<kMaxInlineSegs> k2_fn_n();
