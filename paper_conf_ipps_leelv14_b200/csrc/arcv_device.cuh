@@ -550,22 +550,35 @@ __device__ __forceinline__ uint32_t eval_tile_dispatch(const uint8_t *so, const 
     return eval_tile<T, false, false>(so, sr, si.off_o, si.off_r, si.count, ctid, g, acc);
 }
 
-// DT >= 0: a K1 specialised for one dtype (single-region calls) evaluates only
-// that dtype's tiles; DT < 0: any dtype (batches, tables).
-template <int DT = -1>
+// A K1 specialised for a set of dtypes (bit 1 << ARC_* per dtype) compiles
+// only those dtypes' tile evaluation: one dtype for single-region calls, the
+// set a batch holds (kDtmFloatI32) for batches; kAllDtypes = any region.
+template <int DTM = kAllDtypes>
 __device__ __forceinline__ uint32_t eval_any(const uint8_t *so, const uint8_t *sr, const StageInfo &si, int ctid,
                                              const SegHot &g, ThreadAcc &acc) {
-    if constexpr (DT == ARC_F32) return eval_tile_dispatch<float>(so, sr, si, ctid, g, acc);
-    if constexpr (DT == ARC_F64) return eval_tile_dispatch<double>(so, sr, si, ctid, g, acc);
-    if constexpr (DT == ARC_I32) return eval_tile_dispatch<int32_t>(so, sr, si, ctid, g, acc);
-    if constexpr (DT == ARC_I64) return eval_tile_dispatch<int64_t>(so, sr, si, ctid, g, acc);
-    if constexpr (DT == ARC_U8) return eval_tile_dispatch<uint8_t>(so, sr, si, ctid, g, acc);
-    switch (g.dtype) {
-        case ARC_F32: return eval_tile_dispatch<float>(so, sr, si, ctid, g, acc);
-        case ARC_F64: return eval_tile_dispatch<double>(so, sr, si, ctid, g, acc);
-        case ARC_I32: return eval_tile_dispatch<int32_t>(so, sr, si, ctid, g, acc);
-        case ARC_I64: return eval_tile_dispatch<int64_t>(so, sr, si, ctid, g, acc);
-        default: return eval_tile_dispatch<uint8_t>(so, sr, si, ctid, g, acc);
+    if constexpr (DTM == (1 << ARC_F32)) return eval_tile_dispatch<float>(so, sr, si, ctid, g, acc);
+    else if constexpr (DTM == (1 << ARC_F64)) return eval_tile_dispatch<double>(so, sr, si, ctid, g, acc);
+    else if constexpr (DTM == (1 << ARC_I32)) return eval_tile_dispatch<int32_t>(so, sr, si, ctid, g, acc);
+    else if constexpr (DTM == (1 << ARC_I64)) return eval_tile_dispatch<int64_t>(so, sr, si, ctid, g, acc);
+    else if constexpr (DTM == (1 << ARC_U8)) return eval_tile_dispatch<uint8_t>(so, sr, si, ctid, g, acc);
+    else {
+        switch (g.dtype) {
+            case ARC_F32:
+                if constexpr ((DTM >> ARC_F32) & 1) return eval_tile_dispatch<float>(so, sr, si, ctid, g, acc);
+                else return 0u;  // not launched with this kernel
+            case ARC_F64:
+                if constexpr ((DTM >> ARC_F64) & 1) return eval_tile_dispatch<double>(so, sr, si, ctid, g, acc);
+                else return 0u;
+            case ARC_I32:
+                if constexpr ((DTM >> ARC_I32) & 1) return eval_tile_dispatch<int32_t>(so, sr, si, ctid, g, acc);
+                else return 0u;
+            case ARC_I64:
+                if constexpr ((DTM >> ARC_I64) & 1) return eval_tile_dispatch<int64_t>(so, sr, si, ctid, g, acc);
+                else return 0u;
+            default:
+                if constexpr ((DTM >> ARC_U8) & 1) return eval_tile_dispatch<uint8_t>(so, sr, si, ctid, g, acc);
+                else return 0u;
+        }
     }
 }
 
@@ -1400,7 +1413,7 @@ __global__ void __launch_bounds__(kConsumerThreads) arcv_compact_kernel(const __
 // ------------------------------------------------------------------ K1: stream
 // XF: the sharded exchange is fused into this kernel's tail (its own
 // instantiation, so single-GPU calls carry none of the exchange code).
-template <int S, int MINB, int NSEG, bool XF = false, int DT = -1>
+template <int S, int MINB, int NSEG, bool XF = false, int DTM = kAllDtypes>
 __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __grid_constant__ ParamsN<NSEG> pn) {
     const Params &p = pn;
     extern __shared__ __align__(128) uint8_t smem[];
@@ -1519,7 +1532,7 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
             g.seed_sh = s_red_d;
         }
         const uint8_t *so = smem + (size_t)s * kStageBytes;
-        const uint32_t cnt = (p.flags & kFlagProbe) ? 0u : eval_any<DT>(so, so + kStageArrayBytes, si, ctid, g, acc);
+        const uint32_t cnt = (p.flags & kFlagProbe) ? 0u : eval_any<DTM>(so, so + kStageArrayBytes, si, ctid, g, acc);
         acc.count += cnt;
         if (ctid == 0 && i == 0) ARCV_STAMP(0, 5);
 #if defined(ARCV_TRACE) && ARCV_TRACE

@@ -9,7 +9,7 @@
 namespace arcv {
 
 KernelFnN<1> k1_s3_1_f64(bool xf) {
-    return xf ? arcv_stream_kernel<3, 2, 1, true, ARC_F64> : arcv_stream_kernel<3, 2, 1, false, ARC_F64>;
+    return xf ? arcv_stream_kernel<3, 2, 1, true, (1 << ARC_F64)> : arcv_stream_kernel<3, 2, 1, false, (1 << ARC_F64)>;
 }
 
 }  // namespace arcv

@@ -9,7 +9,7 @@
 namespace arcv {
 
 KernelFnN<1> k1_s3_1_i32(bool xf) {
-    return xf ? arcv_stream_kernel<3, 2, 1, true, ARC_I32> : arcv_stream_kernel<3, 2, 1, false, ARC_I32>;
+    return xf ? arcv_stream_kernel<3, 2, 1, true, (1 << ARC_I32)> : arcv_stream_kernel<3, 2, 1, false, (1 << ARC_I32)>;
 }
 
 }  // namespace arcv

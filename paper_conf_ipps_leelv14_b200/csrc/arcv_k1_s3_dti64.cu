@@ -9,7 +9,7 @@
 namespace arcv {
 
 KernelFnN<1> k1_s3_1_i64(bool xf) {
-    return xf ? arcv_stream_kernel<3, 2, 1, true, ARC_I64> : arcv_stream_kernel<3, 2, 1, false, ARC_I64>;
+    return xf ? arcv_stream_kernel<3, 2, 1, true, (1 << ARC_I64)> : arcv_stream_kernel<3, 2, 1, false, (1 << ARC_I64)>;
 }
 
 }  // namespace arcv

@@ -34,6 +34,8 @@ KernelFnN<1> k1_s3_1_i32(bool xf);
 KernelFnN<1> k1_s3_1_i64(bool xf);
 KernelFnN<1> k1_s3_1_u8(bool xf);
 KernelFnN<1> k1_fn_1_dt(int stages, bool xf, int dtype);  // nullptr: no specialisation
+// K1 with 3 stages for batches of fp32 / fp64 / int32 regions (arcv_k1_s3_dtbatch.cu)
+KernelFnN<kMaxInlineSegs> k1_s3_n_fi();
 // K2 (arcv_k1_s3.cu)
 KernelFnN<1> k2_fn_1();
 KernelFnN<kMaxInlineSegs> k2_fn_n();

@@ -15,6 +15,8 @@ constexpr int kConsumerThreads = kConsumerWarps * 32;
 constexpr int kThreads = kConsumerThreads + 32;     // + producer warp
 constexpr int kVecPerThread = kTileBytes / 16 / kConsumerThreads;  // 4
 constexpr int kMaxInlineSegs = 16;                 // regions passed as kernel parameters (C3: 12)
+constexpr int kAllDtypes = 31;                      // K1 dtype-set masks: bit 1 << ARC_*
+constexpr int kDtmFloatI32 = (1 << ARC_F32) | (1 << ARC_F64) | (1 << ARC_I32);  // batches without i64 / u8
 constexpr int kGroupTiles = 256;                    // tiles per group counter
 constexpr int kPoolCap = 2048;                      // report phase, pool path: max listed nonzero tiles
 #ifndef ARCV_DIRECT_DYN
