@@ -902,3 +902,38 @@ def test_clustered_mismatches_reuse_tiles(av, orc, dt, n_mis):
         gs = av.batch([(out, ref, 1e-6, 1e-5, 1 << 20), (out[te:], ref[te:], 1e-6, 1e-5, 17)])
         assert_same(gs[0], e, f"{dt} batch region 0")
         assert_same(gs[1], orc.compare(on[te:], rn[te:], dt, 1e-6, 1e-5, 17), f"{dt} batch region 1")
+
+
+def test_generic_and_dtype_specialised_k1_agree(orc):
+    """Single-region calls and fp32/fp64/int32 batches run K1s compiled for their dtypes;
+    ARCV_DT_SPEC=0 forces the generic K1 (all dtypes).  Both agree with the oracle, every
+    dtype, aligned and misaligned, single and batched."""
+    import paper_conf_ipps_leelv14_b200 as av
+
+    cases = []
+    for k, dt in enumerate(["f32", "f64", "i32", "i64", "u8"]):
+        n = 3 * TILE_ELEMS[dt] + 101
+        o, r = random_pair(dt, n + 1, 8800 + k, rate=0.002, device="cpu")
+        cases.append((dt, o, r, 0))
+        cases.append((dt, o, r, 1))  # views one element in: misaligned windows
+    expect = [orc.compare(o[off:off + len(o) - 1].numpy(), r[off:off + len(o) - 1].numpy(), dt, 1e-6, 1e-5, 500)
+              for dt, o, r, off in cases]
+    dev = [(dt, o.cuda(), r.cuda(), off) for dt, o, r, off in cases]
+    av.finalize()
+    try:
+        for spec in ("0", "1"):
+            os.environ["ARCV_DT_SPEC"] = spec
+            av.init(0)
+            views = [(o[off:off + o.numel() - 1], r[off:off + r.numel() - 1]) for _, o, r, off in dev]
+            for (dt, _, _, off), (o, r), e in zip(dev, views, expect):
+                assert_same(av.compare(o, r, 1e-6, 1e-5, 500), e, f"spec={spec} {dt} off={off}")
+            fi = [i for i, (dt, _, _, off) in enumerate(dev) if dt in ("f32", "f64", "i32") and off == 0]
+            for i, g in zip(fi, av.batch([(views[i][0], views[i][1], 1e-6, 1e-5, 500) for i in fi])):
+                assert_same(g, expect[i], f"spec={spec} batch {dev[i][0]}")
+            allb = av.batch([(o, r, 1e-6, 1e-5, 500) for o, r in views])
+            for i, g in enumerate(allb):
+                assert_same(g, expect[i], f"spec={spec} mixed batch {i}")
+            av.finalize()
+    finally:
+        del os.environ["ARCV_DT_SPEC"]
+        av.init(0)
