@@ -677,12 +677,15 @@ __device__ __forceinline__ bool last_cta(const Params &p, int tid, int nthreads,
 // completion word needs no system fence -- one PCIe round trip (~3 us) less
 // in the last CTA.  With entries written over PCIe the cumulative system fence
 // orders them (and the slots) before the word.
-__device__ __forceinline__ void publish(const Params &p, int tid, int nthreads, bool fenced = true) {
+// `n_nz`: the launch's final pool length when the caller has it (saves a
+// dependent load on the completion path), else ~0u.
+__device__ __forceinline__ void publish(const Params &p, int tid, int nthreads, bool fenced = true,
+                                        uint32_t n_nz = ~0u) {
     {
         fence_gpu();
         // the report phase's path (the host re-applies direct_route with it)
-        const unsigned long long route =
-            (p.k2 && *(volatile uint32_t *)p.nz_cnt <= (uint32_t)kPoolCap) ? kRoutePool : 0ull;
+        if (n_nz == ~0u) n_nz = *(volatile uint32_t *)p.nz_cnt;
+        const unsigned long long route = (p.k2 && n_nz <= (uint32_t)kPoolCap) ? kRoutePool : 0ull;
         for (uint32_t k = tid; k < p.n_acc; k += nthreads) {
             Acc a;
             a.count = __ldcg(&p.acc[k].count);
@@ -1095,7 +1098,8 @@ constexpr int kReportSmem = 2 * kStageBytes + (int)sizeof(RepShared) + kOutEntri
 
 template <bool XF>
 __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, uint8_t *smem, int tid,
-                                             unsigned long long done_base, bool k1_published_if_empty) {
+                                             unsigned long long done_base, bool k1_published_if_empty,
+                                             uint32_t n_nz_known = ~0u) {
     RepShared &sh = *reinterpret_cast<RepShared *>(smem + 2 * kStageBytes);
     if (tid == 0) {
         ARCV_STAMP(1, 1);
@@ -1152,7 +1156,8 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
         if (tid == 0 && stamp) ARCV_STAMP(1, 2);
     };
 
-    const uint32_t n_nz = *(volatile uint32_t *)p.nz_cnt;
+    // the final pool length: the fused tail read it after the grid barrier already
+    const uint32_t n_nz = n_nz_known != ~0u ? n_nz_known : *(volatile uint32_t *)p.nz_cnt;
     const uint32_t G = gridDim.x, b = blockIdx.x;
     if (n_nz <= (uint32_t)kPoolCap) {
         // ------------------------------------------------------ pool path
@@ -1384,7 +1389,7 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
         // a report kept in device memory (the caller's buffer or HBM staging that
         // the host copies later, stream-ordered) needs no system fence before the
         // completion word: the slots validate themselves (slot_tag)
-        if (last && !(k1_published_if_empty && n_nz == 0)) publish(p, tid, kConsumerThreads, p.report_host != 0);
+        if (last && !(k1_published_if_empty && n_nz == 0)) publish(p, tid, kConsumerThreads, p.report_host != 0, n_nz);
         if constexpr (XF) {
             if (p.xfused) exchange_tail(p, tid, last, smem);
         }
@@ -1605,8 +1610,9 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
             // publishes at once, and no CTA runs the report phase -- each only
             // keeps its counter contract (one grid-barrier arrival, and with
             // `finalize` one done arrival) with fire-and-forget reductions.
-            if (*(volatile uint32_t *)p.nz_cnt == 0u) {
-                if (s_last && p.finalize) publish(p, ctid, kConsumerThreads, false);  // no entry written anywhere
+            const uint32_t n_nz = *(volatile uint32_t *)p.nz_cnt;  // final: every CTA has arrived
+            if (n_nz == 0u) {
+                if (s_last && p.finalize) publish(p, ctid, kConsumerThreads, false, 0u);  // no entry written anywhere
                 if (ctid == 0) {
                     asm volatile("red.relaxed.gpu.global.add.u64 [%0], 1;" ::"l"(p.gbar) : "memory");
                     if (p.finalize) asm volatile("red.relaxed.gpu.global.add.u64 [%0], 1;" ::"l"(p.done) : "memory");
@@ -1616,7 +1622,7 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
                 }
                 return;
             }
-            report_phase<XF>(p, segs, smem, ctid, p.done_base + gridDim.x, true);
+            report_phase<XF>(p, segs, smem, ctid, p.done_base + gridDim.x, true, n_nz);
             return;
         }
     }
