@@ -679,8 +679,11 @@ __device__ __forceinline__ bool last_cta(const Params &p, int tid, int nthreads,
 // orders them (and the slots) before the word.
 // `n_nz`: the launch's final pool length when the caller has it (saves a
 // dependent load on the completion path), else ~0u.
+// `pre` (optional): slot `tid`'s accumulators, already read by the caller after
+// every CTA had flushed (the report phase loads them while its tiles land), so
+// the publishing CTA does not wait for them.
 __device__ __forceinline__ void publish(const Params &p, int tid, int nthreads, bool fenced = true,
-                                        uint32_t n_nz = ~0u) {
+                                        uint32_t n_nz = ~0u, const Acc *pre = nullptr) {
     {
         fence_gpu();
         // the report phase's path (the host re-applies direct_route with it)
@@ -688,9 +691,13 @@ __device__ __forceinline__ void publish(const Params &p, int tid, int nthreads, 
         const unsigned long long route = (p.k2 && n_nz <= (uint32_t)kPoolCap) ? kRoutePool : 0ull;
         for (uint32_t k = tid; k < p.n_acc; k += nthreads) {
             Acc a;
-            a.count = __ldcg(&p.acc[k].count);
-            a.max_abs_bits = __ldcg(&p.acc[k].max_abs_bits);
-            a.max_rel_bits = __ldcg(&p.acc[k].max_rel_bits);
+            if (pre != nullptr && k == (uint32_t)tid) {
+                a = *pre;
+            } else {
+                a.count = __ldcg(&p.acc[k].count);
+                a.max_abs_bits = __ldcg(&p.acc[k].max_abs_bits);
+                a.max_rel_bits = __ldcg(&p.acc[k].max_rel_bits);
+            }
             a.pad = slot_tag(p.seq, route, a.count, a.max_abs_bits, a.max_rel_bits);
             p.result[k] = a;
             if (p.mirror) p.mirror[k] = a;
@@ -1158,6 +1165,15 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
 
     // the final pool length: the fused tail read it after the grid barrier already
     const uint32_t n_nz = n_nz_known != ~0u ? n_nz_known : *(volatile uint32_t *)p.nz_cnt;
+    // this thread's result slot, final since every CTA flushed before the barrier:
+    // read now, off the publishing CTA's critical path
+    Acc pre_acc;
+    const bool have_pre = p.finalize && (uint32_t)tid < p.n_acc;
+    if (have_pre) {
+        pre_acc.count = __ldcg(&p.acc[tid].count);
+        pre_acc.max_abs_bits = __ldcg(&p.acc[tid].max_abs_bits);
+        pre_acc.max_rel_bits = __ldcg(&p.acc[tid].max_rel_bits);
+    }
     const uint32_t G = gridDim.x, b = blockIdx.x;
     if (n_nz <= (uint32_t)kPoolCap) {
         // ------------------------------------------------------ pool path
@@ -1389,7 +1405,8 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
         // a report kept in device memory (the caller's buffer or HBM staging that
         // the host copies later, stream-ordered) needs no system fence before the
         // completion word: the slots validate themselves (slot_tag)
-        if (last && !(k1_published_if_empty && n_nz == 0)) publish(p, tid, kConsumerThreads, p.report_host != 0, n_nz);
+        if (last && !(k1_published_if_empty && n_nz == 0))
+            publish(p, tid, kConsumerThreads, p.report_host != 0, n_nz, have_pre ? &pre_acc : nullptr);
         if constexpr (XF) {
             if (p.xfused) exchange_tail(p, tid, last, smem);
         }
