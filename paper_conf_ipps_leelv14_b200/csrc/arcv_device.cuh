@@ -1375,7 +1375,9 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
                 consumer_bar();
             }
         }
+        if (tid == 0) ARCV_STAMP(1, 3);  // group scan done (trace: "prefixes reduced")
         grid_barrier(p.gbar, p.gbar_base, tid);
+        if (tid == 0) ARCV_STAMP(1, 9);  // active list complete (trace: "pool loaded")
         const uint32_t n_act = *(volatile uint32_t *)p.active_cnt;
         const uint32_t mine = n_act > b ? (n_act - b + G - 1) / G : 0u;
         if (mine > 0 && tid == 0) issue(__ldcg(p.active + 2 * b), 0);
@@ -1384,8 +1386,9 @@ __device__ __forceinline__ void report_phase(const Params &p, const Seg *segs, u
             if (j + 1 < mine && tid == 0) issue(__ldcg(p.active + 2 * (b + (j + 1) * G)), st ^ 1);  // prefetch
             const uint64_t key = __ldcg(p.active + 2 * (b + j * G));
             const uint64_t excl = __ldcg(p.active + 2 * (b + j * G) + 1);
-            emit(key, excl, st, false, 0);
+            emit(key, excl, st, false, 0, j == 0);
         }
+        if (tid == 0) ARCV_STAMP(1, 6);
     }
     // Report entries in pinned host memory need no system-scope fence here:
     // this CTA's gpu-scope release (fence + done counter) is acquired by the
@@ -1583,6 +1586,9 @@ __global__ void __launch_bounds__(kThreads, MINB) arcv_stream_kernel(const __gri
                         // tile that finds the list full lifts it to kPoolCap + 1
                         // (without this, 2049 nonzero tiles could end with a
                         // count of 2048 and take the pool path one tile short).
+                        // (Round 2 measured doing this after the stage release,
+                        // with a per-CTA "pool full" flag: C5 -1 %, C4 +2.2 %,
+                        // profiles/r02s4_ab_late_tile_publish_rejected.log.)
                         const uint32_t v = *(volatile uint32_t *)p.nz_cnt;
                         if (v < (uint32_t)kPoolCap) {
                             const uint32_t k = atomicAdd(p.nz_cnt, 1u);

@@ -77,7 +77,15 @@ def run_probe(name, o, r):
             print(f"  K1 {nm:18s} min {d.min():8.2f}  med {np.median(d):8.2f}  max {d.max():8.2f}  (n={len(col)})")
 
 
-if os.environ.get("TRACE_C2A"):
+if os.environ.get("TRACE_C5"):
+    c5 = synth.C5(1 << int(os.environ.get("TRACE_C5_LOG2", "30")))
+    o, r = c5.slice(device="cuda")
+    rep = torch.empty(24 * c5.max_report, dtype=torch.uint8, device="cuda")
+    res_ = av.arc_verify_result_t()
+    run(f"C5 int32 2^{int(os.environ.get('TRACE_C5_LOG2', '30'))}, 50% mismatches, max_report 2^20 (pinned report)",
+        o, r, 0.0, 0.0, c5.max_report)
+    run("C5, count only", o, r, 0.0, 0.0, 0)
+elif os.environ.get("TRACE_C2A"):
     c2 = synth.C2("A")
     o, r = c2.slice(device="cuda")
     run_probe("read probe over the C2A arrays", o, r)
