@@ -81,7 +81,6 @@ if os.environ.get("TRACE_C5"):
     c5 = synth.C5(1 << int(os.environ.get("TRACE_C5_LOG2", "30")))
     o, r = c5.slice(device="cuda")
     rep = torch.empty(24 * c5.max_report, dtype=torch.uint8, device="cuda")
-    res_ = av.arc_verify_result_t()
     run(f"C5 int32 2^{int(os.environ.get('TRACE_C5_LOG2', '30'))}, 50% mismatches, max_report 2^20 (pinned report)",
         o, r, 0.0, 0.0, c5.max_report)
     run("C5, count only", o, r, 0.0, 0.0, 0)
