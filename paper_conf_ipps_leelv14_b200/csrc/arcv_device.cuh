@@ -114,6 +114,20 @@ constexpr int kTraceCtas = 1024, kTracePts = 32, kTraceRows = 3;
 // [row][cta][point]: row 0 K1, row 1 report phase, row 2 region switches
 // (point 2 seg: switched into segment seg, 2 seg + 1: its first tile evaluated; seg < 16)
 __device__ unsigned long long g_trace[kTraceRows][kTraceCtas][kTracePts];
+// Host side, one per module: merge (element-wise max) this module's stamps into
+// `out` and clear them; the launch that ran stamped only its own module.
+#define ARCV_DEFINE_TRACE_COPY(name)                                                                  \
+    int name(unsigned long long *out, size_t bytes) {                                                 \
+        if (bytes < sizeof(g_trace)) return -1;                                                       \
+        const size_t n = sizeof(g_trace) / 8;                                                         \
+        unsigned long long *tmp = new unsigned long long[n]();                                        \
+        int rc = cudaMemcpyFromSymbol(tmp, g_trace, sizeof(g_trace)) == cudaSuccess ? 0 : -1;         \
+        for (size_t i = 0; rc == 0 && i < n; ++i) out[i] = tmp[i] > out[i] ? tmp[i] : out[i];         \
+        for (size_t i = 0; i < n; ++i) tmp[i] = 0ull;                                                 \
+        if (rc == 0 && cudaMemcpyToSymbol(g_trace, tmp, sizeof(g_trace)) != cudaSuccess) rc = -1;     \
+        delete[] tmp;                                                                                 \
+        return rc;                                                                                    \
+    }
 #define ARCV_STAMP(k, pt)                                                                      \
     do {                                                                                       \
         unsigned long long t_;                                                                 \
@@ -122,6 +136,12 @@ __device__ unsigned long long g_trace[kTraceRows][kTraceCtas][kTracePts];
     } while (0)
 #else
 #define ARCV_STAMP(k, pt) do {} while (0)
+#define ARCV_DEFINE_TRACE_COPY(name)                           \
+    int name(unsigned long long *out, size_t bytes) {          \
+        (void)out;                                             \
+        (void)bytes;                                           \
+        return -1;                                             \
+    }
 #endif
 
 __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {

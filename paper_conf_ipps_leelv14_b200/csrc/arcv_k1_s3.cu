@@ -2,7 +2,6 @@
 // per SM; one translation unit per stage count (arcv_kernels.h).
 #include <cuda_runtime.h>
 
-#include <vector>
 
 #include "arcv_device.cuh"
 #include "arcv_kernels.h"
@@ -17,19 +16,8 @@ KernelFnN<1> k1_s3_1x() { return arcv_stream_kernel<3, 2, 1, true>; }  // sharde
 KernelFnN<1> k2_fn_1() { return arcv_compact_kernel<1>; }
 KernelFnN<kMaxInlineSegs> k2_fn_n() { return arcv_compact_kernel<kMaxInlineSegs>; }
 
-// The trace buffer is a __device__ variable of THIS module (the default K1 and
-// K2); other stage counts are not traced.
-int k1_trace_copy(unsigned long long *out, size_t bytes) {
-#if defined(ARCV_TRACE) && ARCV_TRACE
-    if (bytes < sizeof(g_trace)) return -1;
-    if (cudaMemcpyFromSymbol(out, g_trace, sizeof(g_trace)) != cudaSuccess) return -1;
-    std::vector<unsigned long long> zero(sizeof(g_trace) / 8, 0ull);
-    return cudaMemcpyToSymbol(g_trace, zero.data(), sizeof(g_trace)) == cudaSuccess ? 0 : -1;
-#else
-    (void)out;
-    (void)bytes;
-    return -1;
-#endif
-}
+// The trace buffer is a __device__ variable of each module (translation unit):
+// this one holds the generic K1s and K2, the dtype-specialised K1s have their own.
+ARCV_DEFINE_TRACE_COPY(k1_trace_copy)
 
 }  // namespace arcv

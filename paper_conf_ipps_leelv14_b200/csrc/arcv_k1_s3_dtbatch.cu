@@ -10,4 +10,8 @@ namespace arcv {
 
 KernelFnN<kMaxInlineSegs> k1_s3_n_fi() { return arcv_stream_kernel<3, 2, kMaxInlineSegs, false, kDtmFloatI32>; }
 
+#if defined(ARCV_TRACE) && ARCV_TRACE
+ARCV_DEFINE_TRACE_COPY(k1_trace_copy_batch)
+#endif
+
 }  // namespace arcv

@@ -12,4 +12,8 @@ KernelFnN<1> k1_s3_1_f64(bool xf) {
     return xf ? arcv_stream_kernel<3, 2, 1, true, (1 << ARC_F64)> : arcv_stream_kernel<3, 2, 1, false, (1 << ARC_F64)>;
 }
 
+#if defined(ARCV_TRACE) && ARCV_TRACE
+ARCV_DEFINE_TRACE_COPY(k1_trace_copy_f64)
+#endif
+
 }  // namespace arcv

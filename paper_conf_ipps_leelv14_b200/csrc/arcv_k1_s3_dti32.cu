@@ -12,4 +12,8 @@ KernelFnN<1> k1_s3_1_i32(bool xf) {
     return xf ? arcv_stream_kernel<3, 2, 1, true, (1 << ARC_I32)> : arcv_stream_kernel<3, 2, 1, false, (1 << ARC_I32)>;
 }
 
+#if defined(ARCV_TRACE) && ARCV_TRACE
+ARCV_DEFINE_TRACE_COPY(k1_trace_copy_i32)
+#endif
+
 }  // namespace arcv

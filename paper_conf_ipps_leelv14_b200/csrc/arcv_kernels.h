@@ -41,5 +41,11 @@ KernelFnN<1> k2_fn_1();
 KernelFnN<kMaxInlineSegs> k2_fn_n();
 // ARCV_TRACE builds: copy (and clear) the phase stamps the kernels wrote
 int k1_trace_copy(unsigned long long *out, size_t bytes);
+int k1_trace_copy_f32(unsigned long long *out, size_t bytes);
+int k1_trace_copy_f64(unsigned long long *out, size_t bytes);
+int k1_trace_copy_i32(unsigned long long *out, size_t bytes);
+int k1_trace_copy_i64(unsigned long long *out, size_t bytes);
+int k1_trace_copy_u8(unsigned long long *out, size_t bytes);
+int k1_trace_copy_batch(unsigned long long *out, size_t bytes);
 
 }  // namespace arcv
