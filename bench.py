@@ -93,6 +93,7 @@ class ClockSampler:
         except Exception as e:  # pragma: no cover
             self.err = str(e)
         self._stop = threading.Event()
+        self.interval = 0.005  # seconds between NVML samples
 
     def _run(self):
         while not self._stop.is_set():
@@ -106,7 +107,7 @@ class ClockSampler:
                         self.reasons.add(name)
             except Exception:
                 pass
-            time.sleep(0.005)
+            time.sleep(self.interval)
 
     def __enter__(self):
         if self.ok:
